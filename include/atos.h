@@ -1,0 +1,162 @@
+/*
+ * atos.h -- C ABI of the B200-native Atos hot path (GPU-initiated asynchronous
+ * graph traversal).  Implemented by paper_conf_sc_chenbpbyo22_b200/csrc/ and
+ * built as paper_conf_sc_chenbpbyo22_b200/libatos.so (sm_100a SASS).
+ *
+ * Citations are to /root/reference/PAPER.md (P:<lines>) and the repo's
+ * SURVEY.md §8 / DESIGN.md readings.
+ *
+ * General conventions
+ *  - Every function returns atos_status; no C++ exception crosses the ABI.
+ *    On failure a human-readable message is available from atos_last_error()
+ *    (thread-local, valid until the next ABI call on the same thread).
+ *  - Vertex ids are int32 in [0, n) (n <= 2^31-1); CSR row offsets are int64
+ *    (RMAT-26 symmetric has ~2.1e9 entries; reading R9).
+ *  - Pointer arguments may be HOST or DEVICE memory unless stated otherwise;
+ *    the library inspects them with cudaPointerGetAttributes and copies with
+ *    cudaMemcpyDefault.  Input arrays are caller-owned and only read during
+ *    the call.  Output arrays are caller-owned and caller-allocated.
+ *  - The graph handle owns all device memory it allocates (CSR copy, state,
+ *    queues, channels, control blocks) and frees it in atos_graph_free.
+ *  - A handle is not thread-safe: one host thread drives one handle.
+ */
+#ifndef ATOS_H
+#define ATOS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ATOS_ABI_VERSION 1
+#define ATOS_MAX_RANKS 8          /* one NVSwitch box: 8 GPUs */
+#define ATOS_IPC_HANDLE_BYTES 64  /* == sizeof(cudaIpcMemHandle_t) */
+
+typedef enum {
+    ATOS_OK = 0,
+    ATOS_ERR_INVALID_ARG = 1,  /* bad argument; nothing was modified            */
+    ATOS_ERR_CUDA = 2,         /* a CUDA runtime call failed                    */
+    ATOS_ERR_OOM = 3,          /* device allocation failed                      */
+    ATOS_ERR_CAPACITY = 4,     /* a queue/channel would have overflowed; the
+                                  solve was aborted, outputs are invalid        */
+    ATOS_ERR_TIMEOUT = 5,      /* device watchdog fired; outputs are invalid    */
+    ATOS_ERR_PEER = 6,         /* peer mapping (IPC) failed or is missing       */
+    ATOS_ERR_STATE = 7         /* call not valid in the handle's current state  */
+} atos_status;
+
+typedef struct atos_graph atos_graph;   /* opaque */
+
+/* Launch / runtime configuration.  Obtain defaults with atos_config_init(). */
+typedef struct {
+    int32_t worker_threads;   /* CTA worker size; 512 as in all of the paper's
+                                 runs. Must be 512 in ABI v1.  */
+    int32_t ctas_per_sm;      /* persistent CTAs per SM; 0 = max co-resident */
+    int32_t fetch_size;       /* max vertices popped per worker batch (the
+                                 paper's FETCH_SIZE); <= worker_threads */
+    double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
+    int32_t agg_enabled;      /* communication aggregation on/off */
+    int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */
+    int64_t agg_max_age_ns;   /* flush age (the WAIT_TIME), globaltimer ns     */
+    int32_t channel_packets;  /* packets per (src->dst) channel ring, pow2    */
+    int64_t watchdog_ms;      /* device watchdog per solve; 0 = none           */
+    int32_t rank;             /* SPMD: this process's rank                     */
+    int32_t n_ranks;          /* SPMD: number of processes (1 = single GPU)    */
+    int32_t virtual_ranks;    /* >1 (with n_ranks==1): emulate this many ranks
+                                 inside one grid on one device; same protocol,
+                                 peers are same-device pointers    */
+    int32_t device;           /* CUDA device ordinal                           */
+    void *stream;             /* cudaStream_t to launch on; NULL = the library
+                                 creates its own non-blocking stream           */
+} atos_config;
+
+/* Per-solve statistics (device counters, summed over the ranks this handle
+ * can see; multi-process callers reduce across processes themselves). */
+typedef struct {
+    double ms_worker;         /* device time of the persistent worker kernel
+                                 (CUDA events on the launch stream)           */
+    double ms_total;          /* device time barrier+init+worker+gather        */
+    uint64_t pops;            /* queue entries processed                       */
+    uint64_t edges;           /* edges relaxed (CSR entries scanned)           */
+    uint64_t local_pushes;    /* local ring enqueues                           */
+    uint64_t msgs_sent;       /* remote messages (one-sided peer stores)       */
+    uint64_t packets_sent;    /* channel packets published                     */
+    uint64_t bytes_sent;      /* payload bytes stored into peer channels       */
+    uint64_t idle_polls;      /* worker iterations that found no work          */
+    uint64_t hub_chunks;      /* hub-split edge chunks processed               */
+    int32_t n_ranks;          /* ranks covered by these counters               */
+    int32_t grid_ctas;        /* persistent CTAs per rank                      */
+} atos_stats;
+
+/* Fill *cfg with defaults.  Host only; never touches the GPU. */
+atos_status atos_config_init(atos_config *cfg);
+
+/* 1-D contiguous vertex blocks: part[r] = floor(r*n/p), r = 0..p (SURVEY §8a-1,
+ * reading R13).  part must hold p+1 entries.  Host only. */
+atos_status atos_partition_balanced(int64_t n, int32_t p, int64_t *part);
+
+/* Validate a CSR (row_ptr monotone from 0 to nnz, every col in [0,n)).
+ * row_ptr/col must be HOST pointers.  Host only. */
+atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *col, int64_t n, int64_t nnz);
+
+/* Bytes of the rank-exported device arena for a given shape (host only).
+ * Used by the Python layer to size checks; identical on every rank. */
+atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t n_ranks, int32_t rank,
+                             const atos_config *cfg, uint64_t *bytes_out);
+
+/* Load the graph for this process.  row_ptr [n+1] / col [nnz] describe the
+ * WHOLE directed graph (out-edges, global ids; duplicates and self-loops are
+ * kept as given).  part = n_ranks+1 vertex offsets (NULL = balanced); with
+ * cfg->virtual_ranks = R > 1 the partition has R blocks.  The rank(s) served
+ * by this handle copy only their own rows (Listing 5's CSR + findPE,
+ * P:642-692).  Allocates all device state.  cfg NULL = defaults. */
+atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *col, int64_t n, int64_t nnz,
+                            const int64_t *part, const atos_config *cfg, atos_graph **out);
+
+/* Multi-process (n_ranks > 1) peer mapping, the analogue of nvshmem_malloc's
+ * symmetric heap (Listing 5):  every rank exports one IPC handle for
+ * its arena (ATOS_IPC_HANDLE_BYTES bytes into handle_out), the caller
+ * all-gathers them (torch.distributed), and passes the n_ranks handles in
+ * rank order to atos_graph_connect, which maps every peer over NVLink. */
+atos_status atos_graph_export(atos_graph *g, void *handle_out);
+atos_status atos_graph_connect(atos_graph *g, const void *handles);
+
+/* Asynchronous push BFS from global vertex src (Listing 5,
+ * P:641-699): depth_out[n] receives the hop distance (-1 = unreachable) of
+ * every vertex (all ranks receive the gathered result).  parent_out[n]
+ * (optional, may be NULL) receives the min-id parent (parent[src] = src,
+ * -1 unreachable).  stats optional.  Blocks until the result is in the
+ * output buffers unless all outputs are device pointers and stats == NULL,
+ * in which case it only enqueues on the handle's stream (use atos_sync). */
+atos_status atos_bfs(atos_graph *g, int64_t src, int32_t *depth_out, int64_t *parent_out,
+                     atos_stats *stats);
+
+/* Asynchronous push-residual PageRank: rank = 0,
+ * residual = 1-alpha, every vertex enqueued; pop v -> rank += r, residual
+ * alpha*r/outdeg pushed to each out-neighbour, re-enqueue on the crossing
+ * old < eps <= old+delta (reading R5).  Outputs the raw (unnormalised)
+ * rank_out[n] and residual_out[n] (either may be NULL).  0 <= alpha < 1,
+ * eps > 0.  Same blocking rule as atos_bfs. */
+atos_status atos_pagerank(atos_graph *g, double alpha, double eps, double *rank_out,
+                          double *residual_out, atos_stats *stats);
+
+/* Wait for the last enqueued solve and return its device status. */
+atos_status atos_sync(atos_graph *g);
+
+/* Counters of the last completed solve (synchronises). */
+atos_status atos_last_stats(atos_graph *g, atos_stats *stats);
+
+/* Release everything the handle owns.  NULL-safe. */
+atos_status atos_graph_free(atos_graph *g);
+
+/* Thread-local message describing the last failure on this thread. */
+const char *atos_last_error(void);
+
+/* ABI version (ATOS_ABI_VERSION). */
+int32_t atos_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ATOS_H */

@@ -1,0 +1,678 @@
+// atos.cu -- C ABI (include/atos.h) of the B200-native Atos hot path.
+//
+// Host runtime: graph ingest + 1-D partition, per-rank device
+// arenas (state, ring, channels, control block) laid out identically on every
+// rank so that peers can address each other after IPC mapping (the analogue of
+// NVSHMEM's symmetric heap, Listing 5), kernel launch sequence of
+// one solve (barrier -> init -> persistent worker -> fixup -> gather), error
+// and statistics plumbing.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "../../include/atos.h"
+#include "atos_kernels.cuh"
+
+using namespace atos;
+
+// ---------------------------------------------------------------------------
+// errors
+// ---------------------------------------------------------------------------
+static thread_local char g_err[512] = "";
+
+static atos_status fail(atos_status st, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return st;
+}
+
+#define CU(call)                                                                                  \
+    do {                                                                                          \
+        cudaError_t e_ = (call);                                                                  \
+        if (e_ != cudaSuccess) {                                                                  \
+            return fail(e_ == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA,         \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+        }                                                                                         \
+    } while (0)
+
+extern "C" const char *atos_last_error(void) { return g_err; }
+extern "C" int32_t atos_version(void) { return ATOS_ABI_VERSION; }
+
+// ---------------------------------------------------------------------------
+// config, partition, validation (host only)
+// ---------------------------------------------------------------------------
+extern "C" atos_status atos_config_init(atos_config *cfg) {
+    if (!cfg) return fail(ATOS_ERR_INVALID_ARG, "cfg is NULL");
+    std::memset(cfg, 0, sizeof(*cfg));
+    cfg->worker_threads = kThreads;
+    cfg->ctas_per_sm = 0;
+    cfg->fetch_size = kThreads;
+    cfg->ring_cap_factor = 2.0;
+    cfg->agg_enabled = 1;
+    cfg->agg_batch_msgs = 512;
+    cfg->agg_max_age_ns = 4000;      // ~the paper's eager WAIT_TIME for BFS
+    cfg->channel_packets = 1024;
+    cfg->watchdog_ms = 60000;
+    cfg->rank = 0;
+    cfg->n_ranks = 1;
+    cfg->virtual_ranks = 1;
+    cfg->device = 0;
+    cfg->stream = nullptr;
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_partition_balanced(int64_t n, int32_t p, int64_t *part) {
+    if (n < 0 || p < 1 || p > ATOS_MAX_RANKS || !part)
+        return fail(ATOS_ERR_INVALID_ARG, "partition: need n>=0, 1<=p<=%d, part!=NULL", ATOS_MAX_RANKS);
+    for (int r = 0; r <= p; ++r) part[r] = (int64_t)((__int128)r * n / p);
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *col, int64_t n, int64_t nnz) {
+    if (n < 1 || n > INT32_MAX || nnz < 0 || !row_ptr || (nnz > 0 && !col))
+        return fail(ATOS_ERR_INVALID_ARG, "csr: need 1<=n<=2^31-1, nnz>=0, non-NULL arrays");
+    if (row_ptr[0] != 0 || row_ptr[n] != nnz)
+        return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr[0] must be 0 and row_ptr[n] == nnz");
+    for (int64_t v = 0; v < n; ++v)
+        if (row_ptr[v + 1] < row_ptr[v]) return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone at %lld", (long long)v);
+    for (int64_t e = 0; e < nnz; ++e)
+        if (col[e] < 0 || col[e] >= n) return fail(ATOS_ERR_INVALID_ARG, "csr: col[%lld]=%d out of range", (long long)e, col[e]);
+    return ATOS_OK;
+}
+
+static bool valid_cfg(const atos_config &c) {
+    auto pow2 = [](int64_t x) { return x > 0 && (x & (x - 1)) == 0; };
+    return c.worker_threads == kThreads && c.fetch_size >= 1 && c.fetch_size <= kThreads &&
+           c.ring_cap_factor >= 1.0 && c.agg_batch_msgs >= 1 && c.agg_batch_msgs <= 4096 &&
+           c.agg_max_age_ns >= 0 && pow2(c.channel_packets) && c.channel_packets <= (1 << 20) &&
+           c.watchdog_ms >= 0 && c.n_ranks >= 1 && c.n_ranks <= ATOS_MAX_RANKS && c.rank >= 0 &&
+           c.rank < c.n_ranks && c.virtual_ranks >= 1 && c.virtual_ranks <= ATOS_MAX_RANKS &&
+           !(c.virtual_ranks > 1 && c.n_ranks > 1) && c.ctas_per_sm >= 0 && c.device >= 0;
+}
+
+// ---------------------------------------------------------------------------
+// arena layout: identical computation on every rank
+// ---------------------------------------------------------------------------
+struct Layout {
+    size_t ctrl, depth, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, total;
+    uint64_t ring_cap;
+    int64_t n_r;
+};
+
+static uint64_t pow2_ceil(uint64_t x) {
+    uint64_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+struct Shape {
+    int64_t n;
+    int p;
+    int cp, pkt, stage_cap, ctas_per_rank, fetch;
+    double ring_factor;
+};
+
+static Layout make_layout(const Shape &S, const int64_t *part, int r) {
+    Layout L{};
+    auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
+    L.n_r = part[r + 1] - part[r];
+    L.ring_cap = pow2_ceil(std::max<uint64_t>(1024, (uint64_t)(S.ring_factor * (double)L.n_r) +
+                                                        (uint64_t)S.ctas_per_rank * (uint64_t)S.fetch));
+    size_t o = 0;
+    L.ctrl = o;    o = al(o + sizeof(Ctrl));
+    L.depth = o;   o = al(o + (size_t)S.n * 4);
+    L.rank = o;    o = al(o + (size_t)L.n_r * 8);
+    L.res = o;     o = al(o + (size_t)L.n_r * 8);
+    L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
+    const bool multi = S.p > 1;
+    L.in_hdr = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
+    L.in_pay = o;  o = al(o + (multi ? (size_t)S.p * S.cp * S.pkt * 16 : 0));
+    L.free_m = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
+    L.staging = o; o = al(o + (multi ? (size_t)S.ctas_per_rank * kMaxRanks * S.stage_cap * 16 : 0));
+    L.parent = o;  o = al(o + (size_t)S.n * 8);
+    L.total = o;
+    return L;
+}
+
+static int stage_cap_for(int pkt) { return (int)pow2_ceil((uint64_t)(2 * pkt + kRound)); }
+
+// ---------------------------------------------------------------------------
+// handle
+// ---------------------------------------------------------------------------
+struct LocalRank {
+    int rank = 0;
+    Layout L{};
+    unsigned char *arena = nullptr;
+    int64_t *row_ptr = nullptr;
+    int32_t *col = nullptr;
+    int64_t m_r = 0;
+    uint64_t snap[8] = {0};   // stat counters after the previous solve
+};
+
+struct atos_graph {
+    atos_config cfg{};
+    int64_t n = 0, nnz = 0;
+    int p = 1;          // total ranks (virtual or processes)
+    int n_local = 1;    // ranks served by this handle
+    bool multiproc = false;
+    bool connected = false;
+    std::vector<int64_t> part;
+    Shape S{};
+    int sms = 0, occ = 0, grid = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    LocalRank loc[kMaxRanks];
+    unsigned char *peer_base[kMaxRanks] = {nullptr};
+    bool peer_opened[kMaxRanks] = {false};
+    RankDev *d_ranks = nullptr;
+    int32_t *d_depth_full = nullptr;
+    int64_t **d_accs = nullptr;
+    uint64_t epoch = 0;
+    cudaEvent_t ev_begin = nullptr, ev_w0 = nullptr, ev_w1 = nullptr, ev_end = nullptr;
+    bool pending = false;      // a solve is enqueued but not yet checked
+    atos_stats last{};
+    bool last_valid = false;
+};
+
+template <int APP>
+static cudaError_t kernel_setup(int &occ) {
+    cudaError_t e = cudaFuncSetAttribute(worker_kernel<APP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sizeof(Smem));
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, worker_kernel<APP>, kThreads, sizeof(Smem));
+}
+
+static RankDev build_view(const atos_graph *g, int lr) {
+    const LocalRank &me = g->loc[lr];
+    const int r = me.rank;
+    RankDev d{};
+    d.rank = r;
+    d.n_ranks = g->p;
+    d.n = g->n;
+    d.v_begin = g->part[r];
+    d.v_end = g->part[r + 1];
+    for (int k = 0; k <= kMaxRanks; ++k) d.part[k] = k <= g->p ? g->part[k] : g->n;
+    d.row_ptr = me.row_ptr;
+    d.col = me.col;
+    unsigned char *b = me.arena;
+    const Layout &L = me.L;
+    d.depth = (uint32_t *)(b + L.depth);
+    d.pr_rank = (double *)(b + L.rank);
+    d.pr_res = (double *)(b + L.res);
+    d.ring = (uint64_t *)(b + L.ring);
+    d.ring_cap = L.ring_cap;
+    d.ctrl = (Ctrl *)(b + L.ctrl);
+    const size_t cp = (size_t)g->S.cp, pkt = (size_t)g->S.pkt;
+    d.staging = b + L.staging;
+    d.hubs = nullptr;
+    for (int s = 0; s < g->p; ++s) {
+        // base pointer of rank s's arena as seen from this process
+        unsigned char *bs = nullptr;
+        if (!g->multiproc) bs = g->loc[s].arena;             // virtual ranks / single rank
+        else bs = (s == r) ? b : g->peer_base[s];
+        if (!bs) continue;
+        const Layout Ls = g->multiproc ? make_layout(g->S, g->part.data(), s) : g->loc[s].L;
+        d.peer_ctrl[s] = (Ctrl *)(bs + Ls.ctrl);
+        d.peer_depth[s] = (uint32_t *)(bs + Ls.depth);
+        d.peer_rank[s] = (double *)(bs + Ls.rank);
+        d.peer_res[s] = (double *)(bs + Ls.res);
+        if (g->p > 1) {
+            d.in_hdr[s] = (uint64_t *)(b + L.in_hdr + (size_t)s * cp * 8);
+            d.in_payload[s] = b + L.in_pay + (size_t)s * cp * pkt * 16;
+            d.free_mirror[s] = (uint64_t *)(b + L.free_m + (size_t)s * cp * 8);
+            d.out_hdr[s] = (uint64_t *)(bs + Ls.in_hdr + (size_t)r * cp * 8);
+            d.out_payload[s] = bs + Ls.in_pay + (size_t)r * cp * pkt * 16;
+            d.peer_free[s] = (uint64_t *)(bs + Ls.free_m + (size_t)r * cp * 8);
+        }
+    }
+    return d;
+}
+
+__global__ void rebase_rows_kernel(int64_t *rp, int64_t n1, int64_t base) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n1; i += (int64_t)gridDim.x * blockDim.x)
+        rp[i] -= base;
+}
+
+__global__ void check_rows_kernel(const int64_t *rp, int64_t nr, int64_t m, const int32_t *col, int64_t n,
+                                  unsigned long long *bad) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nr; i += stride)
+        if (rp[i + 1] < rp[i]) atomicOr(bad, 1ull);
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += stride)
+        if (col[e] < 0 || col[e] >= n) atomicOr(bad, 2ull);
+}
+
+__global__ void init_arena_kernel(uint64_t *ring, uint64_t cap, uint64_t *free_m, uint64_t nfree, uint64_t cp) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += stride)
+        ring[i] = pack(lo32(i), 0u);   // free for the producer of index i
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nfree; i += stride)
+        free_m[i] = i % cp;            // packet slot i free for packet index i
+}
+
+static bool is_device_ptr(const void *p) {
+    if (!p) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+static atos_status upload_views(atos_graph *g) {
+    std::vector<RankDev> v(g->n_local);
+    for (int lr = 0; lr < g->n_local; ++lr) v[lr] = build_view(g, lr);
+    CU(cudaMemcpyAsync(g->d_ranks, v.data(), sizeof(RankDev) * g->n_local, cudaMemcpyHostToDevice, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_graph_free(atos_graph *g) {
+    if (!g) return ATOS_OK;
+    cudaSetDevice(g->cfg.device);
+    if (g->stream) cudaStreamSynchronize(g->stream);
+    for (int s = 0; s < kMaxRanks; ++s)
+        if (g->peer_opened[s]) cudaIpcCloseMemHandle(g->peer_base[s]);
+    for (int lr = 0; lr < g->n_local; ++lr) {
+        cudaFree(g->loc[lr].arena);
+        cudaFree(g->loc[lr].row_ptr);
+        cudaFree(g->loc[lr].col);
+    }
+    cudaFree(g->d_ranks);
+    cudaFree(g->d_depth_full);
+    cudaFree(g->d_accs);
+    if (g->ev_begin) cudaEventDestroy(g->ev_begin);
+    if (g->ev_w0) cudaEventDestroy(g->ev_w0);
+    if (g->ev_w1) cudaEventDestroy(g->ev_w1);
+    if (g->ev_end) cudaEventDestroy(g->ev_end);
+    if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+    delete g;
+    return ATOS_OK;
+}
+
+struct GraphGuard {
+    atos_graph *g;
+    ~GraphGuard() { if (g) atos_graph_free(g); }
+};
+
+extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t n_ranks, int32_t rank,
+                                        const atos_config *cfg_in, uint64_t *bytes_out) {
+    atos_config cfg;
+    if (cfg_in) cfg = *cfg_in; else atos_config_init(&cfg);
+    if (!bytes_out || n < 1 || n_ranks < 1 || n_ranks > kMaxRanks || rank < 0 || rank >= n_ranks)
+        return fail(ATOS_ERR_INVALID_ARG, "arena_bytes: bad arguments");
+    std::vector<int64_t> pt(n_ranks + 1);
+    if (part) std::copy(part, part + n_ranks + 1, pt.begin());
+    else atos_partition_balanced(n, n_ranks, pt.data());
+    Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs),
+            148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
+            cfg.fetch_size, cfg.ring_cap_factor};
+    *bytes_out = make_layout(S, pt.data(), rank).total;
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *col, int64_t n, int64_t nnz,
+                                       const int64_t *part, const atos_config *cfg_in, atos_graph **out) {
+    if (!out) return fail(ATOS_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    atos_config cfg;
+    if (cfg_in) cfg = *cfg_in; else atos_config_init(&cfg);
+    if (!valid_cfg(cfg)) return fail(ATOS_ERR_INVALID_ARG, "invalid atos_config");
+    if (!row_ptr || (nnz > 0 && !col) || n < 1 || n > INT32_MAX || nnz < 0)
+        return fail(ATOS_ERR_INVALID_ARG, "graph_load: need 1<=n<=2^31-1, nnz>=0, non-NULL arrays");
+    int ndev = 0;
+    CU(cudaGetDeviceCount(&ndev));
+    if (cfg.device >= ndev) return fail(ATOS_ERR_INVALID_ARG, "device %d not visible (%d devices)", cfg.device, ndev);
+    CU(cudaSetDevice(cfg.device));
+
+    atos_graph *g = new (std::nothrow) atos_graph();
+    if (!g) return fail(ATOS_ERR_OOM, "host allocation failed");
+    GraphGuard guard{g};
+    g->cfg = cfg;
+    g->n = n;
+    g->nnz = nnz;
+    g->multiproc = cfg.n_ranks > 1;
+    g->p = g->multiproc ? cfg.n_ranks : cfg.virtual_ranks;
+    g->n_local = g->multiproc ? 1 : cfg.virtual_ranks;
+    g->part.resize(g->p + 1);
+    if (part) {
+        std::copy(part, part + g->p + 1, g->part.begin());
+        if (g->part[0] != 0 || g->part[g->p] != n)
+            return fail(ATOS_ERR_INVALID_ARG, "part must start at 0 and end at n");
+        for (int r = 0; r < g->p; ++r)
+            if (g->part[r + 1] < g->part[r]) return fail(ATOS_ERR_INVALID_ARG, "part not monotone");
+    } else {
+        atos_partition_balanced(n, g->p, g->part.data());
+    }
+
+    // row offsets at partition boundaries (host copies of a few entries)
+    const bool rp_dev = is_device_ptr(row_ptr);
+    std::vector<int64_t> rb(g->p + 1);
+    for (int r = 0; r <= g->p; ++r) {
+        if (rp_dev) CU(cudaMemcpy(&rb[r], row_ptr + g->part[r], 8, cudaMemcpyDeviceToHost));
+        else rb[r] = row_ptr[g->part[r]];
+    }
+    if (rb[0] != 0 || rb[g->p] != nnz) return fail(ATOS_ERR_INVALID_ARG, "row_ptr[0] must be 0 and row_ptr[n]==nnz");
+
+    // device / occupancy
+    cudaDeviceProp prop;
+    CU(cudaGetDeviceProperties(&prop, cfg.device));
+    g->sms = prop.multiProcessorCount;
+    if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
+    int occ0 = 0, occ1 = 0;
+    CU(kernel_setup<kApBfs>(occ0));
+    CU(kernel_setup<kApPr>(occ1));
+    g->occ = std::min(occ0, occ1);
+    if (cfg.ctas_per_sm > 0) g->occ = std::min(g->occ, cfg.ctas_per_sm);
+    if (g->occ < 1) return fail(ATOS_ERR_CUDA, "worker kernel cannot be resident (occupancy 0)");
+    const int ctas_total = g->occ * g->sms;
+    const int cpr = ctas_total / g->n_local;
+    if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
+    g->grid = cpr * g->n_local;
+    g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs), cpr,
+                 cfg.fetch_size, cfg.ring_cap_factor};
+
+    if (cfg.stream) {
+        g->stream = (cudaStream_t)cfg.stream;
+    } else {
+        CU(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+        g->own_stream = true;
+    }
+    CU(cudaEventCreate(&g->ev_begin));
+    CU(cudaEventCreate(&g->ev_w0));
+    CU(cudaEventCreate(&g->ev_w1));
+    CU(cudaEventCreate(&g->ev_end));
+
+    unsigned long long *d_bad = nullptr;
+    CU(cudaMalloc(&d_bad, sizeof(unsigned long long)));
+    CU(cudaMemsetAsync(d_bad, 0, sizeof(unsigned long long), g->stream));
+    for (int lr = 0; lr < g->n_local; ++lr) {
+        LocalRank &me = g->loc[lr];
+        me.rank = g->multiproc ? cfg.rank : lr;
+        const int r = me.rank;
+        me.L = make_layout(g->S, g->part.data(), r);
+        const int64_t nr = me.L.n_r;
+        me.m_r = rb[r + 1] - rb[r];
+        CU(cudaMalloc(&me.arena, me.L.total));
+        CU(cudaMemsetAsync(me.arena, 0, me.L.total, g->stream));
+        CU(cudaMalloc(&me.row_ptr, (size_t)(nr + 1) * 8));
+        CU(cudaMalloc(&me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
+        CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
+        if (me.m_r > 0)
+            CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
+        rebase_rows_kernel<<<256, 256, 0, g->stream>>>(me.row_ptr, nr + 1, rb[r]);
+        check_rows_kernel<<<1024, 256, 0, g->stream>>>(me.row_ptr, nr, me.m_r, me.col, n, d_bad);
+        const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
+        init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
+                                                       (uint64_t *)(me.arena + me.L.free_m), nfree, g->S.cp);
+        CU(cudaGetLastError());
+    }
+    unsigned long long bad = 0;
+    CU(cudaMemcpyAsync(&bad, d_bad, sizeof(bad), cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    cudaFree(d_bad);
+    if (bad & 1) return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone");
+    if (bad & 2) return fail(ATOS_ERR_INVALID_ARG, "csr: column index out of [0, n)");
+
+    CU(cudaMalloc(&g->d_ranks, sizeof(RankDev) * g->n_local));
+    CU(cudaMalloc(&g->d_depth_full, (size_t)n * 4));
+    CU(cudaMalloc(&g->d_accs, sizeof(int64_t *) * kMaxRanks));
+    g->connected = !g->multiproc;
+    atos_status st = upload_views(g);
+    if (st != ATOS_OK) return st;
+    guard.g = nullptr;
+    *out = g;
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_graph_export(atos_graph *g, void *handle_out) {
+    if (!g || !handle_out) return fail(ATOS_ERR_INVALID_ARG, "export: NULL argument");
+    if (!g->multiproc) return fail(ATOS_ERR_STATE, "export: handle is not multi-process (n_ranks == 1)");
+    CU(cudaSetDevice(g->cfg.device));
+    cudaIpcMemHandle_t h;
+    static_assert(sizeof(h) == ATOS_IPC_HANDLE_BYTES, "IPC handle size");
+    CU(cudaIpcGetMemHandle(&h, g->loc[0].arena));
+    std::memcpy(handle_out, &h, sizeof(h));
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_graph_connect(atos_graph *g, const void *handles) {
+    if (!g || !handles) return fail(ATOS_ERR_INVALID_ARG, "connect: NULL argument");
+    if (!g->multiproc) return fail(ATOS_ERR_STATE, "connect: handle is not multi-process");
+    if (g->connected) return fail(ATOS_ERR_STATE, "connect: already connected");
+    CU(cudaSetDevice(g->cfg.device));
+    const unsigned char *hb = (const unsigned char *)handles;
+    for (int s = 0; s < g->p; ++s) {
+        if (s == g->cfg.rank) { g->peer_base[s] = g->loc[0].arena; continue; }
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, hb + (size_t)s * ATOS_IPC_HANDLE_BYTES, sizeof(h));
+        void *ptr = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess)
+            return fail(ATOS_ERR_PEER, "cudaIpcOpenMemHandle(rank %d) failed: %s", s, cudaGetErrorString(e));
+        g->peer_base[s] = (unsigned char *)ptr;
+        g->peer_opened[s] = true;
+    }
+    g->connected = true;
+    return upload_views(g);
+}
+
+// ---------------------------------------------------------------------------
+// solves
+// ---------------------------------------------------------------------------
+static KParams make_params(atos_graph *g) {
+    KParams kp{};
+    kp.ranks = g->d_ranks;
+    kp.n_local = g->n_local;
+    kp.ctas_per_rank = g->S.ctas_per_rank;
+    kp.fetch = g->cfg.fetch_size;
+    kp.pkt = g->S.pkt;
+    kp.cp = g->S.cp;
+    kp.stage_cap = g->S.stage_cap;
+    kp.agg_on = g->cfg.agg_enabled;
+    kp.n_hub_slots = 0;
+    kp.hub_threshold = INT64_MAX;
+    kp.hub_chunk = 0;
+    kp.agg_age_ns = g->cfg.agg_max_age_ns;
+    kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
+    kp.epoch = g->epoch;
+    return kp;
+}
+
+template <int APP>
+static atos_status launch_worker(atos_graph *g, KParams &kp) {
+    void *args[] = {&kp};
+    CU(cudaLaunchCooperativeKernel((const void *)worker_kernel<APP>, dim3(g->grid), dim3(kThreads), args,
+                                   sizeof(Smem), g->stream));
+    return ATOS_OK;
+}
+
+static atos_status read_ctrl(atos_graph *g, int lr, Ctrl &c) {
+    CU(cudaMemcpy(&c, g->loc[lr].arena + g->loc[lr].L.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost));
+    return ATOS_OK;
+}
+
+// Wait for the enqueued solve, check device error flags, fill g->last.
+static atos_status finish_solve(atos_graph *g) {
+    if (!g->pending) return ATOS_OK;
+    g->pending = false;
+    CU(cudaStreamSynchronize(g->stream));
+    atos_stats st{};
+    st.n_ranks = g->n_local;
+    st.grid_ctas = g->S.ctas_per_rank;
+    float ms = 0;
+    CU(cudaEventElapsedTime(&ms, g->ev_w0, g->ev_w1));
+    st.ms_worker = ms;
+    CU(cudaEventElapsedTime(&ms, g->ev_begin, g->ev_end));
+    st.ms_total = ms;
+    uint64_t err = 0;
+    for (int lr = 0; lr < g->n_local; ++lr) {
+        Ctrl c;
+        atos_status s = read_ctrl(g, lr, c);
+        if (s != ATOS_OK) return s;
+        if (c.error.v && !err) err = c.error.v;
+        const uint64_t now[8] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
+                                 c.st_packets.v, c.st_idle.v, c.st_hub_chunks.v, 0};
+        uint64_t *sn = g->loc[lr].snap;
+        st.pops += now[0] - sn[0];
+        st.edges += now[1] - sn[1];
+        st.local_pushes += now[2] - sn[2];
+        st.msgs_sent += now[3] - sn[3];
+        st.packets_sent += now[4] - sn[4];
+        st.idle_polls += now[5] - sn[5];
+        st.hub_chunks += now[6] - sn[6];
+        std::memcpy(sn, now, sizeof(now));
+    }
+    st.bytes_sent = 0;
+    g->last = st;
+    g->last_valid = true;
+    if (err == kErrCapacity) return fail(ATOS_ERR_CAPACITY, "device queue/channel capacity exceeded; result invalid");
+    if (err == kErrTimeout) return fail(ATOS_ERR_TIMEOUT, "device watchdog (%lld ms) fired; result invalid",
+                                        (long long)g->cfg.watchdog_ms);
+    if (err) return fail(ATOS_ERR_STATE, "device error %llu", (unsigned long long)err);
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_sync(atos_graph *g) {
+    if (!g) return fail(ATOS_ERR_INVALID_ARG, "sync: NULL handle");
+    CU(cudaSetDevice(g->cfg.device));
+    return finish_solve(g);
+}
+
+extern "C" atos_status atos_last_stats(atos_graph *g, atos_stats *stats) {
+    if (!g || !stats) return fail(ATOS_ERR_INVALID_ARG, "last_stats: NULL argument");
+    atos_status s = atos_sync(g);
+    if (s != ATOS_OK && !g->last_valid) return s;
+    if (!g->last_valid) return fail(ATOS_ERR_STATE, "no completed solve");
+    *stats = g->last;
+    return s;
+}
+
+static atos_status begin_solve(atos_graph *g, KParams &kp) {
+    CU(cudaSetDevice(g->cfg.device));
+    if (!g->connected) return fail(ATOS_ERR_PEER, "multi-process handle not connected (atos_graph_connect)");
+    atos_status s = finish_solve(g);   // a previous async solve must be retired first
+    if (s != ATOS_OK) return s;
+    g->epoch++;
+    kp = make_params(g);
+    CU(cudaEventRecord(g->ev_begin, g->stream));
+    if (g->p > 1) barrier_kernel<<<1, 32, 0, g->stream>>>(kp, g->epoch * 4 + 0);
+    return ATOS_OK;
+}
+
+static int grid_for(int64_t n, int threads, int cap) {
+    int64_t b = (n + threads - 1) / threads;
+    return (int)std::max<int64_t>(1, std::min<int64_t>(b, cap));
+}
+
+extern "C" atos_status atos_bfs(atos_graph *g, int64_t src, int32_t *depth_out, int64_t *parent_out,
+                                atos_stats *stats) {
+    if (!g) return fail(ATOS_ERR_INVALID_ARG, "bfs: NULL handle");
+    if (src < 0 || src >= g->n) return fail(ATOS_ERR_INVALID_ARG, "bfs: src %lld not in [0, %lld)", (long long)src, (long long)g->n);
+    if (!depth_out) return fail(ATOS_ERR_INVALID_ARG, "bfs: depth_out is NULL");
+    KParams kp;
+    atos_status s = begin_solve(g, kp);
+    if (s != ATOS_OK) return s;
+    const bool dev_depth = is_device_ptr(depth_out);
+    const bool dev_parent = parent_out && is_device_ptr(parent_out);
+    const int gblocks = g->sms * 4;
+    init_bfs_kernel<<<gblocks, 512, 0, g->stream>>>(kp);
+    seed_bfs_kernel<<<1, 1, 0, g->stream>>>(kp, src);
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(g->ev_w0, g->stream));
+    s = launch_worker<kApBfs>(g, kp);
+    if (s != ATOS_OK) return s;
+    CU(cudaEventRecord(g->ev_w1, g->stream));
+    fixup_kernel<<<1, 512, 0, g->stream>>>(kp);
+    int32_t *dfull = dev_depth ? depth_out : g->d_depth_full;
+    gather_bfs_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(kp, dfull);
+    if (parent_out) {
+        LocalRank &me = g->loc[0];
+        int64_t *acc = (int64_t *)(me.arena + me.L.parent);
+        parent_init_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(acc, g->n);
+        parent_scan_kernel<<<gblocks, 512, 0, g->stream>>>(kp, dfull, acc);
+        int n_acc = 1;
+        int64_t *accs[kMaxRanks];
+        accs[0] = acc;
+        if (g->multiproc) {
+            barrier_kernel<<<1, 32, 0, g->stream>>>(kp, g->epoch * 4 + 1);
+            n_acc = g->p;
+            for (int r = 0; r < g->p; ++r)
+                accs[r] = (int64_t *)(g->peer_base[r] + make_layout(g->S, g->part.data(), r).parent);
+        }
+        CU(cudaMemcpyAsync(g->d_accs, accs, sizeof(int64_t *) * n_acc, cudaMemcpyHostToDevice, g->stream));
+        int64_t *pout = parent_out;
+        int64_t *ptmp = nullptr;
+        if (!dev_parent) {
+            CU(cudaMallocAsync(&ptmp, (size_t)g->n * 8, g->stream));
+            pout = ptmp;
+        }
+        parent_final_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(dfull, g->d_accs, n_acc, g->n,
+                                                                                src, pout);
+        if (!dev_parent) {
+            CU(cudaMemcpyAsync(parent_out, ptmp, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
+            CU(cudaFreeAsync(ptmp, g->stream));
+        }
+    }
+    if (!dev_depth) CU(cudaMemcpyAsync(depth_out, dfull, (size_t)g->n * 4, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(g->ev_end, g->stream));
+    g->pending = true;
+    const bool async = dev_depth && (!parent_out || dev_parent) && !stats;
+    if (async) return ATOS_OK;
+    s = finish_solve(g);
+    if (stats) *stats = g->last;
+    return s;
+}
+
+extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, double *rank_out,
+                                     double *residual_out, atos_stats *stats) {
+    if (!g) return fail(ATOS_ERR_INVALID_ARG, "pagerank: NULL handle");
+    if (!(alpha >= 0.0 && alpha < 1.0)) return fail(ATOS_ERR_INVALID_ARG, "pagerank: alpha must be in [0,1)");
+    if (!(eps > 0.0)) return fail(ATOS_ERR_INVALID_ARG, "pagerank: eps must be > 0");
+    KParams kp;
+    atos_status s = begin_solve(g, kp);
+    if (s != ATOS_OK) return s;
+    kp.alpha = alpha;
+    kp.eps = eps;
+    const int gblocks = g->sms * 4;
+    init_pr_kernel<<<gblocks, 512, 0, g->stream>>>(kp);
+    bump_tail_kernel<<<1, 1, 0, g->stream>>>(kp);
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(g->ev_w0, g->stream));
+    s = launch_worker<kApPr>(g, kp);
+    if (s != ATOS_OK) return s;
+    CU(cudaEventRecord(g->ev_w1, g->stream));
+    fixup_kernel<<<1, 512, 0, g->stream>>>(kp);
+    const bool dev_r = !rank_out || is_device_ptr(rank_out);
+    const bool dev_s = !residual_out || is_device_ptr(residual_out);
+    double *tr = nullptr, *ts = nullptr;
+    if (!dev_r || !dev_s) {
+        // stage through the (idle) parent accumulator region: 8n bytes each is not
+        // guaranteed, so use the full-depth buffer region only for one output.
+        CU(cudaMallocAsync(&tr, (size_t)g->n * 8, g->stream));
+        CU(cudaMallocAsync(&ts, (size_t)g->n * 8, g->stream));
+    }
+    gather_pr_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(
+        kp, rank_out ? (dev_r ? rank_out : tr) : nullptr, residual_out ? (dev_s ? residual_out : ts) : nullptr);
+    if (rank_out && !dev_r) CU(cudaMemcpyAsync(rank_out, tr, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
+    if (residual_out && !dev_s) CU(cudaMemcpyAsync(residual_out, ts, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
+    if (tr) CU(cudaFreeAsync(tr, g->stream));
+    if (ts) CU(cudaFreeAsync(ts, g->stream));
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(g->ev_end, g->stream));
+    g->pending = true;
+    const bool async = dev_r && dev_s && !stats;
+    if (async) return ATOS_OK;
+    s = finish_solve(g);
+    if (stats) *stats = g->last;
+    return s;
+}

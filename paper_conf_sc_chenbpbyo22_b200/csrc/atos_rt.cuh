@@ -1,0 +1,175 @@
+// atos_rt.cuh -- device runtime primitives for the persistent Atos worker.
+//
+// Memory-model wrappers (system/gpu scope acquire/release, fences, globaltimer),
+// the per-rank control block, the device-side rank view, and the lock-free
+// ring queue (Sec. III-A2 + Listing 6) re-designed for
+// sm_100a:  u64 monotone indices, one leader atomic per CTA worker, and
+// self-validating 8-byte slots {seq:32 | item:32} so that publication needs no
+// separate end/end_max/end_count counters (reading R15).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace atos {
+
+constexpr int kMaxRanks = 8;
+constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr int kThreads = 512;   // CTA worker
+constexpr int kWarps = kThreads / 32;
+
+// ---------------------------------------------------------------------------
+// memory model
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_gpu_u32(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t ld_relaxed_sys(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_gpu(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// L2-only (bypass the non-coherent L1) loads for data produced by other SMs/GPUs.
+__device__ __forceinline__ uint64_t ld_cg_u64(const uint64_t *p) { return __ldcg((const unsigned long long *)p); }
+__device__ __forceinline__ uint2 ld_cg_u2(const uint2 *p) { return __ldcg(p); }
+__device__ __forceinline__ uint4 ld_cg_u4(const uint4 *p) { return __ldcg(p); }
+
+__device__ __forceinline__ uint32_t lo32(uint64_t x) { return (uint32_t)x; }
+__device__ __forceinline__ uint32_t hi32(uint64_t x) { return (uint32_t)(x >> 32); }
+__device__ __forceinline__ uint64_t pack(uint32_t hi, uint32_t lo) { return ((uint64_t)hi << 32) | lo; }
+
+// ---------------------------------------------------------------------------
+// control block: every counter on its own 128-byte line
+// ---------------------------------------------------------------------------
+struct alignas(128) Line {
+    uint64_t v;
+    uint64_t pad_[15];
+};
+
+enum DevError : uint64_t { kErrNone = 0, kErrCapacity = 4, kErrTimeout = 5 };
+
+struct Ctrl {
+    Line head;                   // local ring: next index to reserve for pop
+    Line tail;                   // local ring: next index to reserve for push (T)
+    Line finished;               // local ring entries fully processed (F)
+    Line staged;                 // messages sitting in CTA staging buffers
+    Line sent;                   // messages published to peer channels (S)
+    Line recvd;                  // inbound messages fully processed (R)
+    Line done;                   // epoch of the finished solve (set by coordinator)
+    Line error;                  // DevError of the current solve
+    Line started[kMaxRanks];     // [coordinator only] epoch each rank started
+    Line bar[kMaxRanks];         // pre-init barrier arrivals (epoch per rank)
+    Line out_reserve[kMaxRanks]; // packets reserved on channel (this -> d)
+    Line in_cursor[kMaxRanks];   // next packet to consume on channel (s -> this)
+    Line hub_count;              // hub board: number of slots ever claimed
+    Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_chunks, st_waves;
+};
+
+// Per-rank device view.  One per rank served by the grid (virtual ranks: many).
+struct HubSlot {                 // hub work-sharing board entry
+    uint64_t next;               // next edge offset to claim (atomicAdd)
+    uint64_t end;                // row end
+    uint64_t done_edges;         // edges completed (atomicAdd)
+    uint64_t total;              // total edges of the hub  (0 = slot free)
+    uint64_t epoch_tag;          // publication tag (solve epoch<<20 | slot round)
+    uint32_t v;                  // local vertex
+    uint32_t dval_lo, dval_hi;   // app value (depth / delta bits)
+    uint32_t pad_;
+};
+
+struct RankDev {
+    int32_t rank, n_ranks;
+    int64_t n;                   // global vertex count
+    int64_t v_begin, v_end;      // owned global range [v_begin, v_end)
+    int64_t part[kMaxRanks + 1]; // global partition offsets
+    const int64_t *row_ptr;      // [n_r + 1] offsets into col (rank-local rows)
+    const int32_t *col;          // [m_r] global vertex ids
+    // application state (own memory)
+    uint32_t *depth;             // BFS: [n] global-indexed (owned + ghost filter)
+    double *pr_rank;             // PR: [n_r]
+    double *pr_res;              // PR: [n_r]
+    // local ring (own memory)
+    uint64_t *ring;
+    uint64_t ring_cap;           // power of two
+    Ctrl *ctrl;                  // own control block
+    Ctrl *peer_ctrl[kMaxRanks];  // control block of every rank (own included)
+    // channels; a packet = hdr word {seq:32|count:32} + payload of pkt msgs
+    uint64_t *in_hdr[kMaxRanks];       // own memory: inbound from s
+    unsigned char *in_payload[kMaxRanks];
+    uint64_t *out_hdr[kMaxRanks];      // peer memory: d's in_hdr[rank]
+    unsigned char *out_payload[kMaxRanks];
+    uint64_t *free_mirror[kMaxRanks];  // own memory: free tags of packets of channel (this -> d)
+    uint64_t *peer_free[kMaxRanks];    // peer memory: s's free_mirror[rank]
+    // CTA-private staging of outbound messages [cta][dst][stage_cap] (own memory)
+    unsigned char *staging;
+    // hub board (own memory)
+    HubSlot *hubs;
+    // peer state for the final gather
+    uint32_t *peer_depth[kMaxRanks];
+    double *peer_rank[kMaxRanks];
+    double *peer_res[kMaxRanks];
+};
+
+struct KParams {
+    RankDev *ranks;          // device array, one per rank in this grid
+    int32_t n_local;         // ranks served by this grid (virtual ranks)
+    int32_t ctas_per_rank;
+    int32_t fetch;           // vertices per pop batch (<= kThreads)
+    int32_t pkt;             // messages per packet
+    int32_t cp;              // packets per channel (pow2)
+    int32_t stage_cap;       // staging capacity per (cta, dst), messages (pow2)
+    int32_t agg_on;
+    int32_t n_hub_slots;     // pow2
+    int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
+    int64_t hub_chunk;       // edges per hub chunk
+    int64_t agg_age_ns;
+    int64_t watchdog_ns;
+    uint64_t epoch;
+    double alpha, eps;       // PageRank
+};
+
+// ---------------------------------------------------------------------------
+// ring slot encoding (Vyukov-style sequence numbers fused with the item)
+//   free for the producer of index i : seq == lo32(i)
+//   full, item of index i            : seq == lo32(i + 1)
+// consumer of i sets seq = lo32(i + cap) (free for producer of i + cap).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ bool slot_full_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx + 1); }
+__device__ __forceinline__ bool slot_free_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx); }
+
+}  // namespace atos

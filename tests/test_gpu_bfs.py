@@ -1,0 +1,163 @@
+"""GPU parity: asynchronous push BFS (CUDA path through the C ABI) vs the oracle.
+
+Bar (BASELINE.json north_star): depths bit-exact; every GPU parent satisfies
+depth(parent) = depth(v) - 1 via an existing edge (and equals the min-id
+canonical parent the kernel is specified to produce).
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_sc_chenbpbyo22_b200 import atos, inputs
+
+pytestmark = pytest.mark.gpu
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def csr_of(n, edges):
+    edges = sorted(edges)
+    rp = np.zeros(n + 1, dtype=np.int64)
+    for u, _ in edges:
+        rp[u + 1] += 1
+    rp = np.cumsum(rp)
+    col = np.array([v for _, v in edges], dtype=np.int32)
+    return rp, col
+
+
+def check_parents(rp, col, depth, parent, src):
+    n = rp.size - 1
+    assert parent[src] == src
+    assert np.all(parent[depth < 0] == -1)
+    v = np.nonzero((depth > 0))[0]
+    u = parent[v]
+    assert np.all(u >= 0) and np.all(depth[u] == depth[v] - 1)
+    # edge u->v exists
+    for a, b in zip(u[:2000].tolist(), v[:2000].tolist()):
+        assert b in col[rp[a]:rp[a + 1]]
+
+
+def run_and_check(rp, col, src, **cfg):
+    with atos.Graph(rp, col, **cfg) as G:
+        d, par = G.bfs(src, parent=True)
+    want = oracle.bfs(rp, col, src)
+    assert np.array_equal(d, want), f"first diff at {np.nonzero(d != want)[0][:5]}"
+    check_parents(rp, col, d, par, src)
+    assert np.array_equal(par, oracle.bfs_parents_minid(rp, col, want, src))
+    return d
+
+
+def test_hand_fixture_with_self_loops_and_duplicates():
+    fx = json.load(open(os.path.join(GOLDEN, "bfs_hand.json")))
+    rp = np.zeros(len(fx["adj"]) + 1, dtype=np.int64)
+    rp[1:] = np.cumsum([len(a) for a in fx["adj"]])
+    col = np.array([v for a in fx["adj"] for v in a], dtype=np.int32)
+    d = run_and_check(rp, col, fx["src"])
+    assert d.tolist() == fx["depth"]
+
+
+def test_sampled_4_vertex_digraphs():
+    rng = np.random.default_rng(0)
+    pairs = [(u, v) for u in range(4) for v in range(4) if u != v]
+    for mask in rng.choice(1 << 12, 24, replace=False).tolist():
+        edges = [pairs[i] for i in range(12) if mask >> i & 1] or [(0, 1)]
+        rp, col = csr_of(4, edges)
+        run_and_check(rp, col, int(rng.integers(0, 4)))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_small_graphs(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 3000))
+    m = int(rng.integers(1, 6 * n))
+    edges = list(zip(rng.integers(0, n, m).tolist(), rng.integers(0, n, m).tolist()))
+    rp, col = csr_of(n, edges)
+    run_and_check(rp, col, int(rng.integers(0, n)))
+
+
+def test_isolated_source_and_disconnected():
+    rp, col = csr_of(6, [(0, 1), (1, 0), (2, 3), (3, 4)])
+    assert run_and_check(rp, col, 5).tolist() == [-1] * 5 + [0]
+    assert run_and_check(rp, col, 2).tolist() == [-1, -1, 0, 1, 2, -1]
+
+
+def test_long_path_latency_bound():
+    n = 20000
+    rp, col = csr_of(n, [(i, i + 1) for i in range(n - 1)] + [(i + 1, i) for i in range(n - 1)])
+    d = run_and_check(rp, col, 0)
+    assert d[-1] == n - 1
+
+
+def test_kron12_config0_from_vertex0():
+    g = inputs.make_config("kron12")
+    rp, col = g.numpy()
+    run_and_check(rp, col, 0)
+
+
+def test_road_grid_high_diameter():
+    g = inputs.road_grid(300, 200, seed=2)
+    rp, col = g.numpy()
+    run_and_check(rp, col, 0)
+    run_and_check(rp, col, g.n // 2 + 150)
+
+
+def test_repeated_solves_on_one_handle_and_device_outputs():
+    g = inputs.rmat(16, 16, 3, symmetric=True)
+    rp, col = g.numpy()
+    srcs = inputs.bfs_sources(g, 5, seed=3)
+    with atos.Graph(rp, col) as G:
+        for s in srcs:
+            assert np.array_equal(G.bfs(s), oracle.bfs(rp, col, s))
+        out = torch.empty(g.n, dtype=torch.int32, device="cuda")
+        G.bfs(srcs[0], depth_out=out)           # async path: device output
+        G.sync()
+        assert np.array_equal(out.cpu().numpy(), oracle.bfs(rp, col, srcs[0]))
+        st = G.last_stats()
+        assert st["pops"] >= int((out >= 0).sum())
+
+
+@pytest.mark.parametrize("vr", [2, 3, 4, 8])
+@pytest.mark.parametrize("agg", [0, 1])
+def test_virtual_ranks_identical(vr, agg):
+    g = inputs.rmat(15, 16, 1, symmetric=True)
+    rp, col = g.numpy()
+    src = inputs.bfs_sources(g, 1)[0]
+    d = run_and_check(rp, col, src, virtual_ranks=vr, agg_enabled=agg, channel_packets=64)
+    assert (d >= 0).sum() > 1000
+
+
+def test_virtual_ranks_tiny_packets_and_grid_bands():
+    g = inputs.road_grid(120, 100, seed=1)
+    rp, col = g.numpy()
+    run_and_check(rp, col, 0, virtual_ranks=4, agg_batch_msgs=1, channel_packets=2)
+    run_and_check(rp, col, 777, virtual_ranks=8, agg_batch_msgs=7, agg_max_age_ns=0, channel_packets=4)
+
+
+def test_bad_arguments():
+    rp, col = csr_of(3, [(0, 1)])
+    with atos.Graph(rp, col) as G:
+        for bad in (-1, 3):
+            with pytest.raises(atos.AtosError) as e:
+                G.bfs(bad)
+            assert e.value.status == 1
+    with pytest.raises(atos.AtosError):
+        atos.Graph(rp, np.array([7], dtype=np.int32))          # col out of range
+    with pytest.raises(atos.AtosError):
+        atos.Graph(rp, col, device=64)
+
+
+@pytest.mark.slow
+def test_rmat24_config2_full_size():
+    """BASELINE configs[2] at full size, the launch configuration bench.py times."""
+    g = inputs.make_config("rmat24", device="cuda")
+    rp, col = g.row_ptr, g.col
+    srcs = inputs.bfs_sources(g, 2)
+    rpn, coln = g.numpy()
+    with atos.Graph(rp, col) as G:
+        for s in srcs:
+            d = G.bfs(s)
+            want = oracle.bfs(rpn, coln, s)
+            assert np.array_equal(d, want)

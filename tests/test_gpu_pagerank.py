@@ -1,0 +1,112 @@
+"""GPU parity: asynchronous push-residual PageRank vs the oracle (Jacobi to 1e-12).
+
+Bar (BASELINE.json north_star): after normalisation, max per-vertex |err| <= 1e-6
+and L1 err <= 1e-5, fp64 residual accumulation, eps = 1e-9.  Also the
+termination audit: every residual is in [0, eps).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_chenbpbyo22_b200 import atos, inputs
+
+pytestmark = pytest.mark.gpu
+EPS = 1e-9
+ALPHA = 0.85
+
+
+def csr_of(n, edges):
+    edges = sorted(edges)
+    rp = np.zeros(n + 1, dtype=np.int64)
+    for u, _ in edges:
+        rp[u + 1] += 1
+    rp = np.cumsum(rp)
+    col = np.array([v for _, v in edges], dtype=np.int32)
+    return rp, col
+
+
+def run_and_check(rp, col, alpha=ALPHA, eps=EPS, **cfg):
+    with atos.Graph(rp, col, **cfg) as G:
+        rank, res, st = G.pagerank(alpha, eps, stats=True)
+    assert np.all(res >= 0) and np.all(res < eps), "termination audit: residual >= eps left"
+    p_hat = rank / rank.sum()
+    p, _, _ = oracle.pagerank(rp, col, alpha, 1e-12)
+    err = np.abs(p_hat - p)
+    assert err.max() <= 1e-6 and err.sum() <= 1e-5, (err.max(), err.sum())
+    # the bound implied by the readings: ||p_hat - p||_1 <= 2 eps / (1-alpha)^2
+    assert err.sum() <= 2 * eps / (1 - alpha) ** 2 + 1e-10
+    return p_hat, st
+
+
+def test_cycle_uniform():
+    n = 1000
+    rp, col = csr_of(n, [(i, (i + 1) % n) for i in range(n)])
+    p_hat, _ = run_and_check(rp, col)
+    assert np.allclose(p_hat, 1.0 / n, atol=1e-9)
+
+
+def test_star_closed_form():
+    k = 5
+    e = [(0, i) for i in range(1, k + 1)] + [(i, 0) for i in range(1, k + 1)]
+    rp, col = csr_of(k + 1, e)
+    p_hat, _ = run_and_check(rp, col)
+    assert abs(p_hat[0] - 5.25 / 11.1) < 1e-8
+
+
+def test_all_dangling_and_single_vertex():
+    rp, col = csr_of(7, [])
+    run_and_check(rp, col)
+    rp, col = csr_of(1, [])
+    run_and_check(rp, col)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_random_with_dangling_selfloops_multiedges(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 4000))
+    m = int(rng.integers(0, 8 * n))
+    edges = list(zip(rng.integers(0, n, m).tolist(), rng.integers(0, n, m).tolist()))
+    rp, col = csr_of(n, edges)
+    run_and_check(rp, col, alpha=float(rng.choice([0.5, 0.85])))
+
+
+def test_rmat14_directed():
+    g = inputs.rmat(14, 16, 2, symmetric=False)
+    rp, col = g.numpy()
+    _, st = run_and_check(rp, col)
+    assert st["pops"] >= g.n
+
+
+@pytest.mark.parametrize("vr", [2, 4, 8])
+@pytest.mark.parametrize("agg", [0, 1])
+def test_virtual_ranks(vr, agg):
+    g = inputs.rmat(13, 16, 1, symmetric=False)
+    rp, col = g.numpy()
+    run_and_check(rp, col, virtual_ranks=vr, agg_enabled=agg, channel_packets=64)
+
+
+def test_repeated_solves_one_handle():
+    g = inputs.rmat(12, 16, 4, symmetric=False)
+    rp, col = g.numpy()
+    p, _, _ = oracle.pagerank(rp, col, ALPHA, 1e-12)
+    with atos.Graph(rp, col) as G:
+        for _ in range(3):
+            rank, res = G.pagerank(ALPHA, EPS)
+            assert np.abs(rank / rank.sum() - p).sum() <= 1e-5
+
+
+def test_bad_arguments():
+    rp, col = csr_of(3, [(0, 1)])
+    with atos.Graph(rp, col) as G:
+        for a, e in [(1.0, 1e-9), (-0.1, 1e-9), (0.85, 0.0), (0.85, float("nan"))]:
+            with pytest.raises(atos.AtosError) as ex:
+                G.pagerank(a, e)
+            assert ex.value.status == 1
+
+
+@pytest.mark.slow
+def test_rmat20_config1_full_size():
+    """BASELINE configs[1]: RMAT-20 ef16 directed, alpha .85, eps 1e-9, 1 GPU."""
+    g = inputs.make_config("rmat20_pr", device="cuda")
+    rp, col = g.numpy()
+    run_and_check(g.row_ptr, g.col)
