@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""bench.py -- BFS & PageRank GTEPS of the B200-native Atos hot path.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl atos|reference] [--workload NAME]
+
+Headline (BASELINE.json metric, configs[2]): asynchronous push BFS on RMAT-24
+ef16 (symmetrised), 1-D vertex partition over N GPUs (strong scaling), one step
+= one BFS solve (barrier, init, persistent worker, termination, gather) from
+the next of 16 sampled non-isolated sources.  value = sum of m_reached over the
+K timed steps / device time (max over ranks), in GTEPS, m_reached = directed
+CSR entries of reached vertices (reading R23).  The PageRank line of
+the metric (configs[1], RMAT-20 directed, alpha .85, eps 1e-9) is reported
+under "pagerank".  Inputs are seeded synthetic graphs generated on the device;
+the CSR (2.2 GB) is larger than L2 (126 MB), so no L2 flush is done between
+steps (said in config.l2).
+
+--impl reference times the CPU oracle (oracle/, test infrastructure) on the
+same workload: each step is one serial BFS from that step's source.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_sc_chenbpbyo22_b200 import dist as adist  # noqa: E402
+from paper_conf_sc_chenbpbyo22_b200 import inputs  # noqa: E402
+
+WORKLOADS = {
+    "bfs_rmat24": ("rmat24", "bfs"),
+    "bfs_rmat26": ("rmat26", "bfs"),
+    "bfs_kron12": ("kron12", "bfs"),
+    "bfs_grid4900": ("grid4900", "bfs"),
+}
+KERNELS_PER_BFS_STEP = {1: 5}    # init, seed, worker, fixup, gather (+ barrier when N > 1)
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, STREAM-style copy)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        self.lines = []
+        if self.proc is not None:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [l for l in out.splitlines() if l.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in getattr(self, "lines", []):
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_graph(name: str, device):
+    t0 = time.time()
+    g = inputs.make_config(name, device=device)
+    log(f"[bench] generated {g.name}: n={g.n} nnz={g.nnz} in {time.time() - t0:.1f}s on {device}")
+    return g
+
+
+def m_reached_of(depth_dev: torch.Tensor, deg: torch.Tensor):
+    reached = depth_dev >= 0
+    return int(deg[reached].sum().item()), int(reached.sum().item())
+
+
+def cpu_baseline_bfs(g, src: int, m_reached: int):
+    import oracle
+    rp, col = g.row_ptr.cpu().numpy(), g.col.cpu().numpy()
+    t0 = time.perf_counter()
+    d = oracle.bfs(rp, col, src)
+    dt = time.perf_counter() - t0
+    return {"value": m_reached / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"1 serial FIFO BFS (oracle/oracle.c) from source {src} on the full {g.name} graph, "
+                      f"{dt:.2f} s on 1 host core", "seconds": dt, "reached": int((d >= 0).sum())}
+
+
+def run_reference(args, rank, world):
+    """Reference arm = the CPU oracle, timed as it stands on the box's host cores."""
+    if rank != 0:
+        return
+    import oracle
+    gname, app = WORKLOADS[args.workload]
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    g = make_graph(gname, dev)
+    srcs = [0] if gname == "kron12" else inputs.bfs_sources(g, args.sources)
+    rp, col = g.row_ptr.cpu().numpy(), g.col.cpu().numpy()
+    deg = np.diff(rp)
+    for k in range(args.warmup):
+        oracle.bfs(rp, col, srcs[k % len(srcs)])
+    edges = 0
+    t0 = time.perf_counter()
+    for k in range(args.steps):
+        d = oracle.bfs(rp, col, srcs[(args.warmup + k) % len(srcs)])
+        edges += int(deg[d >= 0].sum())
+    dt = time.perf_counter() - t0
+    v = edges / dt / 1e9
+    line = {"impl": "reference", "metric": "BFS GTEPS (RMAT, 1-D partition) -- CPU oracle",
+            "value": v, "unit": "GTEPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "i32", "data": "synthetic",
+            "config": {"workload": f"{args.workload}", "graph": g.name, "n": g.n, "nnz": g.nnz,
+                       "sources": len(srcs)},
+            "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} serial FIFO BFS solves (oracle/oracle.c) on the full graph"},
+            "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=16)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="atos", choices=["atos", "reference"])
+    ap.add_argument("--workload", default="bfs_rmat24", choices=sorted(WORKLOADS))
+    ap.add_argument("--sources", type=int, default=16)
+    ap.add_argument("--pr-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-pr", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--agg", type=int, default=1)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("[bench] warmup raised to 3 (timing rule)")
+        args.warmup = 3
+
+    rank, world, local = adist.init()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    assert torch.cuda.is_available(), "bench.py (impl atos) needs a CUDA device; no CPU fallback"
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_sc_chenbpbyo22_b200 import atos
+
+    gname, app = WORKLOADS[args.workload]
+    g = make_graph(gname, dev)
+    deg = g.degrees()
+    srcs = [0] if gname == "kron12" else inputs.bfs_sources(g, args.sources)
+    stream = torch.cuda.current_stream(dev)
+    cfg = dict(agg_enabled=args.agg, stream=stream.cuda_stream)
+    if world > 1:
+        G = adist.load_distributed(g.row_ptr, g.col, g.n, **cfg)
+    else:
+        G = atos.Graph(g.row_ptr, g.col, g.n, **cfg)
+    depth = torch.empty(g.n, dtype=torch.int32, device=dev)
+
+    # units per source (computed once from the device result; counting only)
+    units = {}
+    for s in srcs:
+        G.bfs(s, depth_out=depth)
+        G.sync()
+        units[s] = m_reached_of(depth, deg)
+
+    for k in range(args.warmup):
+        G.bfs(srcs[k % len(srcs)], depth_out=depth)
+        G.last_stats()
+
+    seq = [srcs[(args.warmup + k) % len(srcs)] for k in range(args.steps)]
+    worker_ms, edges_scanned, pops = [], 0, 0
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for s in seq:
+            G.bfs(s, depth_out=depth)
+            st = G.last_stats()          # retires the solve (sync + error check), no extra device work
+            worker_ms.append(st["ms_worker"])
+            edges_scanned += st["edges"]
+            pops += st["pops"]
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    ms_rank = ev0.elapsed_time(ev1)
+    ms = adist.max_over_ranks(ms_rank)
+    m_total = sum(units[s][0] for s in seq)
+    n_total = sum(units[s][1] for s in seq)
+    value = m_total / (ms * 1e-3) / 1e9
+
+    # roofline of the dominant kernel (the persistent worker), SURVEY §8d byte model
+    peak, peak_src = peaks()
+    bytes_per_launch = (8 * m_total + 28 * n_total) / len(seq) / world
+    avg_worker_ms = adist.max_over_ranks(sum(worker_ms) / len(worker_ms))
+    achieved = bytes_per_launch / (avg_worker_ms * 1e-3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_worker_traffic.json")
+    if os.path.exists(prof):
+        try:
+            pj = json.load(open(prof))
+            if pj.get("workload") == args.workload:
+                traffic = pj.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic, "kernel": "atos::worker_kernel<BFS>", "peak_source": peak_src,
+            "bytes_model": "8*m_reached + 28*n_reached per BFS (SURVEY 8d)",
+            "worker_ms_avg": avg_worker_ms, "worker_share_of_step": avg_worker_ms / (ms / len(seq))}
+
+    line = {"metric": "BFS & PageRank GTEPS (max over ranks); headline = BFS GTEPS",
+            "value": value, "unit": "GTEPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms / len(seq), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (seeded Graph500 RMAT, device-generated)",
+            "config": {"workload": args.workload, "graph": g.name, "n": g.n, "nnz": g.nnz,
+                       "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
+                       "aggregation": bool(args.agg),
+                       "l2": "no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9)},
+            "gpu_launches": args.steps * (KERNELS_PER_BFS_STEP[1] + (1 if world > 1 else 0)),
+            "roofline": roof,
+            "counters": {"pops_per_reached": pops / max(1, n_total), "edges_per_m_reached": edges_scanned / max(1, m_total)}}
+    line["clocks"] = clk.summary()
+
+    # ---- e2e: through the public API from pinned host memory, every step:
+    # H2D of the CSR (graph_load), BFS, D2H of the depth array, free.
+    rp_h = g.row_ptr.cpu().pin_memory()
+    col_h = g.col.cpu().pin_memory()
+    depth_h = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    if args.e2e_steps > 0:
+        e_units = 0
+        if world > 1:
+            torch.distributed.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for k in range(args.e2e_steps):
+            s = seq[k % len(seq)]
+            if world > 1:
+                H = adist.load_distributed(rp_h, col_h, g.n, **cfg)
+            else:
+                H = atos.Graph(rp_h, col_h, g.n, **cfg)
+            H.bfs(s, depth_out=depth_h)
+            H.free()
+            e_units += units[s][0]
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e_ms = adist.max_over_ranks(e0.elapsed_time(e1))
+        line["e2e"] = {"value": e_units / (e_ms * 1e-3) / 1e9, "unit": "GTEPS",
+                       "h2d_bytes_per_step": int((g.n + 1) * 8 + g.nnz * 4),
+                       "d2h_bytes_per_step": int(g.n * 4), "steps": args.e2e_steps,
+                       "what": "atos_graph_load(pinned host CSR) + atos_bfs(host depth out) + atos_graph_free per step"}
+        # query-only variant: graph resident, source in, host depth out
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        qu = 0
+        for s in seq[:4]:
+            G.bfs(s, depth_out=depth_h)
+            qu += units[s][0]
+        q1.record(stream)
+        torch.cuda.synchronize()
+        q_ms = adist.max_over_ranks(q0.elapsed_time(q1))
+        line["e2e_query"] = {"value": qu / (q_ms * 1e-3) / 1e9, "unit": "GTEPS", "h2d_bytes_per_step": 8,
+                             "d2h_bytes_per_step": int(g.n * 4),
+                             "what": "graph resident; atos_bfs(src) -> pinned host depth"}
+
+    # ---- PageRank line of the metric (configs[1])
+    if not args.no_pr and world == 1:
+        gp = make_graph("rmat20_pr", dev)
+        P = atos.Graph(gp.row_ptr, gp.col, gp.n, **cfg)
+        r_out = torch.empty(gp.n, dtype=torch.float64, device=dev)
+        s_out = torch.empty(gp.n, dtype=torch.float64, device=dev)
+        P.pagerank(0.85, 1e-9, rank_out=r_out, residual_out=s_out)
+        P.last_stats()
+        torch.cuda.synchronize()
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        relax, pr_pops, pr_worker = 0, 0, []
+        p0.record(stream)
+        for _ in range(args.pr_steps):
+            P.pagerank(0.85, 1e-9, rank_out=r_out, residual_out=s_out)
+            st = P.last_stats()
+            relax += st["edges"]
+            pr_pops += st["pops"]
+            pr_worker.append(st["ms_worker"])
+        p1.record(stream)
+        torch.cuda.synchronize()
+        p_ms = p0.elapsed_time(p1) / args.pr_steps
+        line["pagerank"] = {"workload": "pr_rmat20 (configs[1]) alpha=0.85 eps=1e-9", "graph": gp.name,
+                            "n": gp.n, "nnz": gp.nnz, "ms_per_solve": p_ms,
+                            "gteps_relaxations": relax / args.pr_steps / (p_ms * 1e-3) / 1e9,
+                            "gteps_nnz_per_solve": gp.nnz / (p_ms * 1e-3) / 1e9,
+                            "relaxations_per_nnz": relax / args.pr_steps / gp.nnz,
+                            "pops_per_vertex": pr_pops / args.pr_steps / gp.n,
+                            "worker_ms_avg": sum(pr_worker) / len(pr_worker), "dtype": "f64"}
+        P.free()
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only)
+    if not args.no_cpu_baseline and world == 1 and rank == 0:
+        s = seq[0]
+        line["cpu_baseline"] = cpu_baseline_bfs(g, s, units[s][0])
+
+    G.free()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

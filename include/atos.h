@@ -55,6 +55,13 @@ typedef struct {
     int32_t ctas_per_sm;      /* persistent CTAs per SM; 0 = max co-resident */
     int32_t fetch_size;       /* max vertices popped per worker batch (the
                                  paper's FETCH_SIZE); <= worker_threads */
+    int32_t keep_items;       /* max discovered vertices a worker keeps as its
+                                 own next batch when the ring is nearly empty
+                                 (work-keeping; 0 = always enqueue); <= 512    */
+    int32_t l2_persist;       /* 1: give the random-access state (BFS words /
+                                 PR residuals) an L2 persisting access-policy
+                                 window during the worker kernel; sets the
+                                 device's persisting-L2 limit to its maximum  */
     double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
     int32_t agg_enabled;      /* communication aggregation on/off */
     int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */
@@ -85,6 +92,8 @@ typedef struct {
     uint64_t bytes_sent;      /* payload bytes stored into peer channels       */
     uint64_t idle_polls;      /* worker iterations that found no work          */
     uint64_t hub_chunks;      /* hub-split edge chunks processed               */
+    uint64_t busy_ns;         /* sum over workers of time spent on work (ns)   */
+    uint64_t batches;         /* work units (pop batches + packets + chunks)   */
     int32_t n_ranks;          /* ranks covered by these counters               */
     int32_t grid_ctas;        /* persistent CTAs per rank                      */
 } atos_stats;

@@ -9,7 +9,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libatos.so")
 SOURCES = [os.path.join(CSRC, "atos.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("atos_rt.cuh", "atos_kernels.cuh")] + \
+DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("atos_rt.cuh", "atos_worker.cuh", "atos_aux.cuh")] + \
     [os.path.join(ROOT, "include", "atos.h")]
 
 NVCC_FLAGS = [

@@ -32,6 +32,8 @@ class Config(ctypes.Structure):
         ("worker_threads", ctypes.c_int32),
         ("ctas_per_sm", ctypes.c_int32),
         ("fetch_size", ctypes.c_int32),
+        ("keep_items", ctypes.c_int32),
+        ("l2_persist", ctypes.c_int32),
         ("ring_cap_factor", ctypes.c_double),
         ("agg_enabled", ctypes.c_int32),
         ("agg_batch_msgs", ctypes.c_int32),
@@ -58,6 +60,8 @@ class Stats(ctypes.Structure):
         ("bytes_sent", ctypes.c_uint64),
         ("idle_polls", ctypes.c_uint64),
         ("hub_chunks", ctypes.c_uint64),
+        ("busy_ns", ctypes.c_uint64),
+        ("batches", ctypes.c_uint64),
         ("n_ranks", ctypes.c_int32),
         ("grid_ctas", ctypes.c_int32),
     ]

@@ -16,7 +16,8 @@
 #include <vector>
 
 #include "../../include/atos.h"
-#include "atos_kernels.cuh"
+#include "atos_aux.cuh"
+#include "atos_worker.cuh"
 
 using namespace atos;
 
@@ -54,9 +55,11 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->worker_threads = kThreads;
     cfg->ctas_per_sm = 0;
     cfg->fetch_size = kThreads;
+    cfg->keep_items = 0;
+    cfg->l2_persist = 1;
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
-    cfg->agg_batch_msgs = 512;
+    cfg->agg_batch_msgs = 256;
     cfg->agg_max_age_ns = 4000;      // ~the paper's eager WAIT_TIME for BFS
     cfg->channel_packets = 1024;
     cfg->watchdog_ms = 60000;
@@ -90,6 +93,7 @@ extern "C" atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *
 static bool valid_cfg(const atos_config &c) {
     auto pow2 = [](int64_t x) { return x > 0 && (x & (x - 1)) == 0; };
     return c.worker_threads == kThreads && c.fetch_size >= 1 && c.fetch_size <= kThreads &&
+           c.keep_items >= 0 && c.keep_items <= kThreads &&
            c.ring_cap_factor >= 1.0 && c.agg_batch_msgs >= 1 && c.agg_batch_msgs <= 4096 &&
            c.agg_max_age_ns >= 0 && pow2(c.channel_packets) && c.channel_packets <= (1 << 20) &&
            c.watchdog_ms >= 0 && c.n_ranks >= 1 && c.n_ranks <= ATOS_MAX_RANKS && c.rank >= 0 &&
@@ -135,13 +139,13 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.in_hdr = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
     L.in_pay = o;  o = al(o + (multi ? (size_t)S.p * S.cp * S.pkt * 16 : 0));
     L.free_m = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
-    L.staging = o; o = al(o + (multi ? (size_t)S.ctas_per_rank * kMaxRanks * S.stage_cap * 16 : 0));
+    L.staging = o; o = al(o + (multi ? (size_t)S.ctas_per_rank * kWarps * kMaxRanks * S.stage_cap * 16 : 0));
     L.parent = o;  o = al(o + (size_t)S.n * 8);
     L.total = o;
     return L;
 }
 
-static int stage_cap_for(int pkt) { return (int)pow2_ceil((uint64_t)(2 * pkt + kRound)); }
+static int stage_cap_for(int pkt) { return (int)pow2_ceil((uint64_t)std::max(2 * pkt, 64)); }
 
 // ---------------------------------------------------------------------------
 // handle
@@ -153,7 +157,7 @@ struct LocalRank {
     int64_t *row_ptr = nullptr;
     int32_t *col = nullptr;
     int64_t m_r = 0;
-    uint64_t snap[8] = {0};   // stat counters after the previous solve
+    uint64_t snap[9] = {0};   // stat counters after the previous solve
 };
 
 struct atos_graph {
@@ -166,6 +170,7 @@ struct atos_graph {
     std::vector<int64_t> part;
     Shape S{};
     int sms = 0, occ = 0, grid = 0;
+    size_t persist_max = 0, window_max = 0;   // L2 persisting-cache limits of the device
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     LocalRank loc[kMaxRanks];
@@ -177,6 +182,7 @@ struct atos_graph {
     uint64_t epoch = 0;
     cudaEvent_t ev_begin = nullptr, ev_w0 = nullptr, ev_w1 = nullptr, ev_end = nullptr;
     bool pending = false;      // a solve is enqueued but not yet checked
+    int app = kApBfs;          // application of the pending / last solve
     atos_stats last{};
     bool last_valid = false;
 };
@@ -366,6 +372,16 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     cudaDeviceProp prop;
     CU(cudaGetDeviceProperties(&prop, cfg.device));
     g->sms = prop.multiProcessorCount;
+    g->persist_max = (size_t)prop.persistingL2CacheMaxSize;
+    g->window_max = (size_t)prop.accessPolicyMaxWindowSize;
+    if (cfg.l2_persist && g->persist_max > 0) {
+        size_t cur = 0;
+        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+        if (cur < g->persist_max && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, g->persist_max) != cudaSuccess) {
+            cudaGetLastError();
+            g->persist_max = 0;   // not permitted here: run without the window
+        }
+    }
     if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
     int occ0 = 0, occ1 = 0;
     CU(kernel_setup<kApBfs>(occ0));
@@ -478,6 +494,7 @@ static KParams make_params(atos_graph *g) {
     kp.cp = g->S.cp;
     kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
+    kp.keep = g->cfg.keep_items;
     kp.n_hub_slots = 0;
     kp.hub_threshold = INT64_MAX;
     kp.hub_chunk = 0;
@@ -489,9 +506,34 @@ static KParams make_params(atos_graph *g) {
 
 template <int APP>
 static atos_status launch_worker(atos_graph *g, KParams &kp) {
-    void *args[] = {&kp};
-    CU(cudaLaunchCooperativeKernel((const void *)worker_kernel<APP>, dim3(g->grid), dim3(kThreads), args,
-                                   sizeof(Smem), g->stream));
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3(g->grid);
+    lc.blockDim = dim3(kThreads);
+    lc.dynamicSmemBytes = sizeof(Smem);
+    lc.stream = g->stream;
+    cudaLaunchAttribute at[2];
+    int na = 0;
+    at[na].id = cudaLaunchAttributeCooperative;          // co-residency of the persistent grid
+    at[na].val.cooperative = 1;
+    ++na;
+    if (g->cfg.l2_persist && g->n_local == 1 && g->persist_max > 0 && g->window_max > 0) {
+        // keep the random-access state (BFS words / PR residuals) resident in L2
+        // while the CSR column stream passes through
+        const LocalRank &me = g->loc[0];
+        void *base = APP == kApBfs ? (void *)(me.arena + me.L.depth) : (void *)(me.arena + me.L.res);
+        size_t bytes = APP == kApBfs ? (size_t)g->n * 4 : (size_t)me.L.n_r * 8;
+        bytes = std::min(bytes, g->window_max);
+        at[na].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[na].val.accessPolicyWindow.base_ptr = base;
+        at[na].val.accessPolicyWindow.num_bytes = bytes;
+        at[na].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)g->persist_max / (double)bytes);
+        at[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        ++na;
+    }
+    lc.attrs = at;
+    lc.numAttrs = na;
+    CU(cudaLaunchKernelEx(&lc, worker_kernel<APP>, kp));
     return ATOS_OK;
 }
 
@@ -501,7 +543,10 @@ static atos_status read_ctrl(atos_graph *g, int lr, Ctrl &c) {
 }
 
 // Wait for the enqueued solve, check device error flags, fill g->last.
+static constexpr int kSnap = 9;
+
 static atos_status finish_solve(atos_graph *g) {
+    const int app = g->app;
     if (!g->pending) return ATOS_OK;
     g->pending = false;
     CU(cudaStreamSynchronize(g->stream));
@@ -519,8 +564,9 @@ static atos_status finish_solve(atos_graph *g) {
         atos_status s = read_ctrl(g, lr, c);
         if (s != ATOS_OK) return s;
         if (c.error.v && !err) err = c.error.v;
-        const uint64_t now[8] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
-                                 c.st_packets.v, c.st_idle.v, c.st_hub_chunks.v, 0};
+        const uint64_t now[kSnap] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
+                                     c.st_packets.v, c.st_idle.v, c.st_hub_chunks.v, c.st_busy_ns.v,
+                                     c.st_batches.v};
         uint64_t *sn = g->loc[lr].snap;
         st.pops += now[0] - sn[0];
         st.edges += now[1] - sn[1];
@@ -529,9 +575,12 @@ static atos_status finish_solve(atos_graph *g) {
         st.packets_sent += now[4] - sn[4];
         st.idle_polls += now[5] - sn[5];
         st.hub_chunks += now[6] - sn[6];
+        st.busy_ns += now[7] - sn[7];
+        st.batches += now[8] - sn[8];
         std::memcpy(sn, now, sizeof(now));
     }
-    st.bytes_sent = 0;
+    st.bytes_sent = st.msgs_sent * (uint64_t)(app == kApBfs ? AppTraits<kApBfs>::kMsgBytes
+                                                            : AppTraits<kApPr>::kMsgBytes);
     g->last = st;
     g->last_valid = true;
     if (err == kErrCapacity) return fail(ATOS_ERR_CAPACITY, "device queue/channel capacity exceeded; result invalid");
@@ -626,6 +675,7 @@ extern "C" atos_status atos_bfs(atos_graph *g, int64_t src, int32_t *depth_out, 
     CU(cudaGetLastError());
     CU(cudaEventRecord(g->ev_end, g->stream));
     g->pending = true;
+    g->app = kApBfs;
     const bool async = dev_depth && (!parent_out || dev_parent) && !stats;
     if (async) return ATOS_OK;
     s = finish_solve(g);
@@ -670,6 +720,7 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     CU(cudaGetLastError());
     CU(cudaEventRecord(g->ev_end, g->stream));
     g->pending = true;
+    g->app = kApPr;
     const bool async = dev_r && dev_s && !stats;
     if (async) return ATOS_OK;
     s = finish_solve(g);

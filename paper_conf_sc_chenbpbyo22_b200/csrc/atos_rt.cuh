@@ -13,7 +13,16 @@
 namespace atos {
 
 constexpr int kMaxRanks = 8;
-constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr uint32_t kInf = 0xFFFFFFFFu;        // BFS word of an undiscovered vertex
+constexpr uint32_t kDepthInf = 0x7FFFFFFFu;   // its depth field
+
+// BFS per-vertex word: (depth << 1) | pending.  `pending` is set by every
+// improving atomicMin and cleared (atomicAnd) by the one pop that expands the
+// vertex at that depth, so stale duplicate queue entries are skipped without a
+// second array.  Ordering by the word == ordering by depth for improvements:
+// atomicMin(w, dw(nd)) > dw(nd)  <=>  depth(w) > nd.
+__device__ __forceinline__ uint32_t dw_make(uint32_t d) { return (d << 1) | 1u; }
+__device__ __forceinline__ uint32_t dw_depth(uint32_t w) { return w >> 1; }
 constexpr int kThreads = 512;   // CTA worker
 constexpr int kWarps = kThreads / 32;
 
@@ -97,7 +106,9 @@ struct Ctrl {
     Line out_reserve[kMaxRanks]; // packets reserved on channel (this -> d)
     Line in_cursor[kMaxRanks];   // next packet to consume on channel (s -> this)
     Line hub_count;              // hub board: number of slots ever claimed
+    Line ring_base;              // tail at the start of the current solve
     Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_chunks, st_waves;
+    Line st_busy_ns, st_batches;
 };
 
 // Per-rank device view.  One per rank served by the grid (virtual ranks: many).
@@ -120,7 +131,7 @@ struct RankDev {
     const int64_t *row_ptr;      // [n_r + 1] offsets into col (rank-local rows)
     const int32_t *col;          // [m_r] global vertex ids
     // application state (own memory)
-    uint32_t *depth;             // BFS: [n] global-indexed (owned + ghost filter)
+    uint32_t *depth;             // BFS: [n] global-indexed words dw (owned + ghost filter)
     double *pr_rank;             // PR: [n_r]
     double *pr_res;              // PR: [n_r]
     // local ring (own memory)
@@ -152,8 +163,9 @@ struct KParams {
     int32_t fetch;           // vertices per pop batch (<= kThreads)
     int32_t pkt;             // messages per packet
     int32_t cp;              // packets per channel (pow2)
-    int32_t stage_cap;       // staging capacity per (cta, dst), messages (pow2)
+    int32_t stage_cap;       // staging capacity per (cta, warp, dst), messages (pow2)
     int32_t agg_on;
+    int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
     int32_t n_hub_slots;     // pow2
     int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
     int64_t hub_chunk;       // edges per hub chunk
@@ -171,5 +183,9 @@ struct KParams {
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ bool slot_full_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx + 1); }
 __device__ __forceinline__ bool slot_free_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx); }
+
+__device__ __forceinline__ void set_error(const RankDev &R, uint64_t code) {
+    atomicCAS((unsigned long long *)&R.ctrl->error.v, 0ull, (unsigned long long)code);
+}
 
 }  // namespace atos

@@ -1,0 +1,762 @@
+// atos_worker.cuh -- the persistent Atos worker for sm_100a.
+//
+// One CTA of 512 threads is one Atos "worker".
+// The grid is persistent and co-resident (cooperative launch), one process per
+// GPU; with virtual ranks, several ranks share one grid (blockIdx -> rank).
+//
+// Worker loop (Listing 3):
+//   1. every warp tries to claim one ready inbound packet from a peer channel
+//      and applies it (owner-side atomicMin / atomicAdd; enqueue if improved /
+//      crossed)
+//   2. otherwise the CTA pops a batch of <= fetch vertices from the local ring
+//      (reserve-then-wait, one leader atomic per worker) and
+//      expands it: the batch's edge space is cut into 256-edge chunks that the
+//      16 warps process independently (no block barrier inside the edge loop),
+//      8 edges per lane in flight:
+//        BFS (Listing 5): probe depth[u], atomicMin if it
+//          would improve, enqueue u if it did;
+//        PR: atomicAdd alpha*r/outdeg into res[u],
+//          enqueue on the crossing old < eps <= old+delta.
+//      Local discoveries go to per-warp shared-memory staging; remote ones to
+//      per-warp message staging that warps publish to the owner's channel as
+//      packets with one-sided stores over NVLink (aggregation by size / age,
+//      PAPER.md:995-1065).  At batch end the CTA enqueues its discoveries with
+//      one leader atomic, or keeps up to `keep` of them as its next batch when
+//      the ring is nearly empty (work-keeping chain: latency-bound graphs never
+//      round-trip through the queue).
+//   3. idle: flush aged staging, termination detection (single rank: F == T;
+//      multi-rank: coordinator double wave), watchdog.
+#pragma once
+#include "atos_rt.cuh"
+
+namespace atos {
+
+constexpr int kApBfs = 0;
+constexpr int kApPr = 1;
+constexpr int kU = 8;                // edges per lane in flight
+constexpr int kChunk = 32 * kU;      // edges per warp chunk
+constexpr int kWOut = 256;           // per-warp local staging (items)
+constexpr uint32_t kFull = 0xffffffffu;
+
+template <int APP> struct AppTraits;
+template <> struct AppTraits<kApBfs> { static constexpr int kMsgBytes = 8; };
+template <> struct AppTraits<kApPr> { static constexpr int kMsgBytes = 16; };
+
+struct Smem {
+    RankDev R;
+    uint32_t v[kThreads];          // batch: local vertex ids
+    uint64_t val[kThreads];        // batch: depth (BFS) or delta bits (PR)
+    int64_t beg[kThreads];         // batch: row begin (offset into col)
+    int64_t off[kThreads + 1];     // batch: exclusive prefix of edge counts
+    uint32_t wout[kWarps][kWOut];  // per-warp local push staging
+    uint32_t wn[kWarps];
+    uint32_t wpre[kWarps + 1];
+    uint32_t chunk_next;           // next unclaimed edge chunk of the batch
+    uint32_t wst[kWarps][kMaxRanks], wsh[kWarps][kMaxRanks];   // per-warp message staging tail/head
+    uint64_t wt0[kWarps][kMaxRanks];                           // time staging became non-empty
+    int64_t wsum[kWarps];
+    uint64_t res_lo, res_hi;       // outstanding ring reservation
+    uint64_t ring_base;            // ring tail at the start of this solve
+    uint64_t b64[4];
+    int32_t b32[4];
+    int32_t minbad;
+    int32_t flag;
+    uint64_t staged_reported;
+    uint64_t wave[kMaxRanks][5];   // coordinator double wave
+    int32_t wave_valid;
+    unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
+};
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+__device__ __forceinline__ int owner_of(const RankDev &R, int64_t u) {
+    int r = 0;
+#pragma unroll
+    for (int k = 1; k < kMaxRanks; ++k) r += (k < R.n_ranks && R.part[k] <= u) ? 1 : 0;
+    return r;
+}
+
+// Streaming loads of the column array: bypass L1, evict-first in L2 so that the
+// random-access state (depth / residual) stays L2-resident.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ int32_t ld_stream(const int32_t *ptr, uint64_t pol) {
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
+    return v;
+}
+
+// Block-wide exclusive scan of one int64 per thread; returns the total.
+__device__ __forceinline__ int64_t block_exscan(Smem &s, int64_t x, int64_t &excl) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int64_t incl = x;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const int64_t y = __shfl_up_sync(kFull, incl, d);
+        if (lane >= d) incl += y;
+    }
+    if (lane == 31) s.wsum[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+        const int64_t t = lane < kWarps ? s.wsum[lane] : 0;
+        int64_t ti = t;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const int64_t y = __shfl_up_sync(kFull, ti, d);
+            if (lane >= d) ti += y;
+        }
+        if (lane < kWarps) s.wsum[lane] = ti - t;
+        if (lane == kWarps - 1) s.b64[3] = (uint64_t)ti;
+    }
+    __syncthreads();
+    excl = incl - x + s.wsum[w];
+    const int64_t total = (int64_t)s.b64[3];
+    __syncthreads();
+    return total;
+}
+
+// largest j in [lo, hi] with off[j] <= e   (off[lo] <= e holds)
+__device__ __forceinline__ int upper_vertex(const Smem &s, int lo, int hi, int64_t e) {
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (s.off[mid] <= e) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+// ---------------------------------------------------------------------------
+// local ring pushes
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void ring_store(const RankDev &R, uint64_t idx, uint32_t item, uint64_t base) {
+    uint64_t *p = &R.ring[idx & (R.ring_cap - 1)];
+    uint32_t spins = 0;
+    // every index below the solve's base was consumed or retired, so slots of the
+    // first lap of this solve are free without looking; later laps check the tag
+    while (idx - base >= R.ring_cap && !slot_free_for(ld_relaxed_gpu(p), idx)) {
+        if (++spins > (1u << 24)) { set_error(R, kErrCapacity); return; }
+        __nanosleep(64);
+    }
+    st_relaxed_gpu(p, pack(lo32(idx + 1), item));
+}
+
+// Whole warp: push wout[w][0..wn) with one leader atomic.
+__device__ void warp_flush_local(Smem &s, int w, uint32_t &wn) {
+    __syncwarp();
+    const uint32_t cnt = wn;
+    if (cnt == 0) return;
+    const int lane = threadIdx.x & 31;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd((unsigned long long *)&s.R.ctrl->tail.v, (unsigned long long)cnt);
+    base = __shfl_sync(kFull, base, 0);
+    fence_acq_rel_gpu();   // release this warp's state updates before the items become visible
+    for (uint32_t i = lane; i < cnt; i += 32) ring_store(s.R, base + i, s.wout[w][i], s.ring_base);
+    if (lane == 0) atomicAdd(&s.c_pushes, (unsigned long long)cnt);
+    wn = 0;
+    __syncwarp();
+}
+
+// Whole warp: lanes with pred append item (caller guarantees wn + 32 <= kWOut).
+__device__ __forceinline__ void warp_append_local(Smem &s, int w, uint32_t &wn, bool pred, uint32_t item) {
+    const uint32_t m = __ballot_sync(kFull, pred);
+    if (pred) s.wout[w][wn + __popc(m & lanemask_lt())] = item;
+    wn += __popc(m);
+}
+
+// ---------------------------------------------------------------------------
+// remote messages: per-warp staging per destination; packets over NVLink
+// ---------------------------------------------------------------------------
+template <int APP>
+__device__ __forceinline__ unsigned char *wstage(const Smem &s, const KParams &kp, int cta, int w, int d) {
+    const size_t slot = (((size_t)cta * kWarps + w) * kMaxRanks + d) * (size_t)kp.stage_cap;
+    return s.R.staging + slot * AppTraits<APP>::kMsgBytes;
+}
+
+template <int APP> __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn);
+
+// Whole warp: publish `cnt` staged messages for dst as one packet.
+template <int APP>
+__device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int d, uint32_t cnt, uint32_t &wn) {
+    const RankDev &R = s.R;
+    const int lane = threadIdx.x & 31;
+    const uint32_t cp = (uint32_t)kp.cp;
+    unsigned long long pidx = 0;
+    if (lane == 0) pidx = atomicAdd((unsigned long long *)&R.ctrl->out_reserve[d].v, 1ull);
+    pidx = __shfl_sync(kFull, pidx, 0);
+    const uint32_t slot = (uint32_t)(pidx & (cp - 1));
+    uint64_t t_begin = 0;
+    for (;;) {   // wait for the receiver to free the slot; keep consuming inbound meanwhile
+        int st = 0;
+        if (lane == 0) {
+            const uint64_t f = ld_acquire_sys(&R.free_mirror[d][slot]);
+            if (lo32(f) == lo32(pidx)) st = 1;
+            else {
+                const uint64_t now = globaltimer();
+                if (t_begin == 0) t_begin = now;
+                if (ld_relaxed_gpu(&R.ctrl->error.v) != 0 || now - t_begin > 4000000000ull) {
+                    set_error(R, kErrCapacity);
+                    st = 2;
+                }
+            }
+        }
+        st = __shfl_sync(kFull, st, 0);
+        if (st == 1) break;
+        if (st == 2) return false;
+        warp_inbound<APP>(s, kp, w, wn);
+    }
+    const unsigned char *src = wstage<APP>(s, kp, cta, w, d);
+    const uint32_t h = s.wsh[w][d];
+    const uint32_t mask = (uint32_t)(kp.stage_cap - 1);
+    unsigned char *dpay = R.out_payload[d] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+    for (uint32_t i = lane; i < cnt; i += 32) {     // coalesced one-sided stores into d's HBM
+        const uint32_t q = (h + i) & mask;
+        if constexpr (APP == kApBfs) ((uint64_t *)dpay)[i] = ((const uint64_t *)src)[q];
+        else ((uint4 *)dpay)[i] = ((const uint4 *)src)[q];
+    }
+    __threadfence_system();
+    __syncwarp();
+    if (lane == 0) {
+        atomicAdd((unsigned long long *)&R.ctrl->sent.v, (unsigned long long)cnt);   // S before publish
+        fence_acq_rel_sys();
+        st_release_sys(&R.out_hdr[d][slot], pack(lo32(pidx + 1), cnt));
+        s.wsh[w][d] = h + cnt;
+        if (s.wsh[w][d] == s.wst[w][d]) s.wt0[w][d] = 0;
+        atomicAdd(&s.c_msgs, (unsigned long long)cnt);
+        atomicAdd(&s.c_packets, 1ull);
+    }
+    __syncwarp();
+    return true;
+}
+
+// Whole warp: send full packets (and partial ones when `partial`) for every destination.
+template <int APP>
+__device__ void warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t &wn) {
+    const RankDev &R = s.R;
+    if (R.n_ranks <= 1) return;
+    const uint64_t now = globaltimer();
+    for (int d = 0; d < R.n_ranks; ++d) {
+        if (d == R.rank) continue;
+        for (;;) {
+            __syncwarp();
+            const uint32_t pending = s.wst[w][d] - s.wsh[w][d];
+            if (pending == 0) break;
+            bool go = pending >= (uint32_t)kp.pkt;
+            if (!go && batch_end) {
+                const uint64_t t0 = s.wt0[w][d];
+                go = !kp.agg_on || (t0 != 0 && now - t0 >= (uint64_t)kp.agg_age_ns);
+            }
+            go = __shfl_sync(kFull, go, 0);
+            if (!go) break;
+            const uint32_t cnt = pending < (uint32_t)kp.pkt ? pending : (uint32_t)kp.pkt;
+            if (!warp_send_packet<APP>(s, kp, cta, w, d, cnt, wn)) return;
+        }
+    }
+}
+
+// Whole warp: lanes with pred stage a message (dst, v_local at dst, payload).
+template <int APP>
+__device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, int cta, int w, bool pred, int dst,
+                                                   uint32_t v_local, uint64_t payload, uint32_t &wn) {
+    const RankDev &R = s.R;
+    if (__ballot_sync(kFull, pred) == 0) return;
+    const int lane = threadIdx.x & 31;
+    const uint32_t mask = (uint32_t)(kp.stage_cap - 1);
+    for (int d = 0; d < R.n_ranks; ++d) {
+        const bool mine = pred && dst == d;
+        const uint32_t m = __ballot_sync(kFull, mine);
+        if (m == 0) continue;
+        __syncwarp();
+        if (s.wst[w][d] - s.wsh[w][d] + 32 > (uint32_t)kp.stage_cap) {
+            // full packets out first (keeps room for this row)
+            warp_flush_remote<APP>(s, kp, cta, w, false, wn);
+            __syncwarp();
+        }
+        const uint32_t t = s.wst[w][d];
+        if (mine) {
+            unsigned char *b = wstage<APP>(s, kp, cta, w, d);
+            const uint32_t pos = (t + __popc(m & lanemask_lt())) & mask;
+            if constexpr (APP == kApBfs) ((uint64_t *)b)[pos] = pack((uint32_t)payload, v_local);
+            else ((uint4 *)b)[pos] = make_uint4(v_local, 0u, (uint32_t)payload, (uint32_t)(payload >> 32));
+        }
+        __syncwarp();
+        if (lane == 0) {
+            if (t == s.wsh[w][d]) s.wt0[w][d] = globaltimer();
+            s.wst[w][d] = t + __popc(m);
+        }
+        __syncwarp();
+    }
+}
+
+// Whole warp: claim one ready inbound packet and apply it (owner-side receive).
+template <int APP>
+__device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
+    const RankDev &R = s.R;
+    if (R.n_ranks <= 1) return false;
+    const int lane = threadIdx.x & 31;
+    const uint32_t cp = (uint32_t)kp.cp;
+    int src = -1;
+    uint32_t cnt = 0;
+    unsigned long long c = 0;
+    if (lane == 0) {
+        const int p = R.n_ranks;
+        const int start = (w + (int)(s.c_idle & 7)) % p;
+        for (int k = 0; k < p; ++k) {
+            const int sr = (start + k) % p;
+            if (sr == R.rank) continue;
+            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[sr].v;
+            const uint64_t cc = ld_relaxed_gpu((const uint64_t *)cur);
+            const uint64_t h = ld_acquire_sys(&R.in_hdr[sr][cc & (cp - 1)]);
+            if (hi32(h) == lo32(cc + 1) && atomicCAS(cur, cc, cc + 1) == cc) {
+                src = sr;
+                cnt = lo32(h);
+                c = cc;
+                break;
+            }
+        }
+    }
+    src = __shfl_sync(kFull, src, 0);
+    if (src < 0) return false;
+    cnt = __shfl_sync(kFull, cnt, 0);
+    c = __shfl_sync(kFull, c, 0);
+    const uint32_t slot = (uint32_t)(c & (cp - 1));
+    const unsigned char *pay = R.in_payload[src] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+    for (uint32_t base = 0; base < cnt; base += 32) {
+        const uint32_t i = base + lane;
+        bool pred = false;
+        uint32_t ul = 0;
+        if (i < cnt) {
+            if constexpr (APP == kApBfs) {
+                const uint64_t m = ld_cg_u64((const uint64_t *)pay + i);
+                ul = lo32(m);
+                const uint32_t ndw = dw_make(hi32(m));
+                pred = atomicMin(R.depth + R.v_begin + ul, ndw) > ndw;
+            } else {
+                const uint4 m = ld_cg_u4((const uint4 *)pay + i);
+                ul = m.x;
+                const double dlt = __longlong_as_double((long long)(((uint64_t)m.w << 32) | m.z));
+                const double old = atomicAdd(R.pr_res + ul, dlt);
+                pred = old < kp.eps && old + dlt >= kp.eps;
+            }
+        }
+        if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+        warp_append_local(s, w, wn, pred, ul);
+    }
+    warp_flush_local(s, w, wn);             // T counts the new local work before R
+    if (lane == 0) {
+        st_release_sys(&R.peer_free[src][slot], c + cp);   // slot free for the sender
+        fence_acq_rel_sys();
+        atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)cnt);
+    }
+    __syncwarp();
+    return true;
+}
+
+// ---------------------------------------------------------------------------
+// batch expansion
+// ---------------------------------------------------------------------------
+template <int APP>
+__device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
+    const RankDev &R = s.R;
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t vb = R.v_begin, ve = R.v_end;
+    const bool multi = R.n_ranks > 1;
+    const uint64_t pol = policy_evict_first();
+    const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
+    int jprev = 0;
+    for (;;) {
+        // dynamic chunk claim: a warp that finishes early takes the next chunk
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(&s.chunk_next, 1u);
+        c = __shfl_sync(kFull, c, 0);
+        if (c >= nch) break;
+        const int64_t c0 = (int64_t)c * kChunk;
+        const int64_t clast = (E < c0 + kChunk ? E : c0 + kChunk) - 1;
+        const int jlo = upper_vertex(s, s.off[jprev] <= c0 ? jprev : 0, B - 1, c0);
+        const int jhi = upper_vertex(s, jlo, B - 1, clast);
+        jprev = jlo;
+        int j = jlo;
+        int32_t u[kU];
+        uint64_t vv[kU];
+#pragma unroll
+        for (int k = 0; k < kU; ++k) {
+            const int64_t e = c0 + k * 32 + lane;
+            u[k] = -1;
+            vv[k] = 0;
+            if (e <= clast) {
+                if (j < jhi && s.off[j + 1] <= e) {       // usually one step for skewed graphs
+                    ++j;
+                    if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
+                }
+                u[k] = ld_stream(R.col + s.beg[j] + (e - s.off[j]), pol);
+                vv[k] = s.val[j];
+            }
+        }
+        if constexpr (APP == kApBfs) {
+            uint32_t cur[kU];
+#pragma unroll
+            for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? R.depth[u[k]] : 0u;   // probe (stale = larger: safe)
+            bool imp[kU];
+#pragma unroll
+            for (int k = 0; k < kU; ++k) {
+                const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
+                imp[k] = false;
+                if (u[k] >= 0 && ndw < cur[k]) imp[k] = atomicMin(R.depth + u[k], ndw) > ndw;
+            }
+#pragma unroll
+            for (int k = 0; k < kU; ++k) {
+                const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
+                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+                warp_append_local(s, w, wn, loc, (uint32_t)(u[k] - vb));
+                if (multi) {
+                    const bool rem = imp[k] && !loc;
+                    const int d = rem ? owner_of(R, u[k]) : 0;
+                    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
+                                            (uint64_t)((uint32_t)vv[k] + 1u), wn);
+                }
+            }
+        } else {
+            const double eps = kp.eps;
+            bool cross[kU];
+#pragma unroll
+            for (int k = 0; k < kU; ++k) {
+                cross[k] = false;
+                if (u[k] >= vb && u[k] < ve) {
+                    const double dlt = __longlong_as_double((long long)vv[k]);
+                    const double old = atomicAdd(R.pr_res + (u[k] - vb), dlt);
+                    cross[k] = old < eps && old + dlt >= eps;        // crossing enqueue (R5)
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < kU; ++k) {
+                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+                warp_append_local(s, w, wn, cross[k], (uint32_t)(u[k] - vb));
+                if (multi) {
+                    const bool rem = u[k] >= 0 && !(u[k] >= vb && u[k] < ve);
+                    const int d = rem ? owner_of(R, u[k]) : 0;
+                    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u, vv[k], wn);
+                }
+            }
+        }
+    }
+}
+
+// Load per-vertex info of the batch s.v[0..B) and expand it.
+template <int APP>
+__device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
+    const RankDev &R = s.R;
+    const int tid = threadIdx.x;
+    int64_t deg = 0;
+    if (tid < B) {
+        const uint32_t v = s.v[tid];
+        const int64_t b = R.row_ptr[v], e = R.row_ptr[v + 1];
+        s.beg[tid] = b;
+        deg = e - b;
+        if constexpr (APP == kApBfs) {
+            // claim the expansion of v at its current depth; stale duplicates see
+            // the pending bit already cleared and are skipped
+            const uint32_t old = atomicAnd(R.depth + R.v_begin + v, ~1u);
+            const uint32_t d = dw_depth(old);
+            s.val[tid] = d;
+            if (!(old & 1u) || d == kDepthInf) deg = 0;
+        } else {
+            const double r = __longlong_as_double(
+                (long long)atomicExch((unsigned long long *)(R.pr_res + v), 0ull));
+            if (r != 0.0) atomicAdd(R.pr_rank + v, r);
+            if (r == 0.0 || deg == 0) deg = 0;        // dangling vertices absorb (R4)
+            else s.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
+        }
+    }
+    int64_t excl;
+    const int64_t E = block_exscan(s, deg, excl);
+    if (tid < B) s.off[tid] = excl;
+    if (tid == 0) { s.off[B] = E; s.c_edges += (unsigned long long)E; s.chunk_next = 0; }
+    __syncthreads();
+    if (E > 0) {
+        const int w = tid >> 5;
+        uint32_t wn = s.wn[w];
+        expand_warp<APP>(s, kp, cta, B, E, wn);
+        __syncwarp();
+        if ((tid & 31) == 0) s.wn[w] = wn;
+    }
+}
+
+// End of a batch: publish remote staging per policy, then enqueue this CTA's
+// local discoveries with one leader atomic -- or keep up to kp.keep of them as
+// the next batch (returned count, already in s.v) when the ring is nearly empty.
+template <int APP>
+__device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
+    const int tid = threadIdx.x, w = tid >> 5;
+    __syncthreads();
+    if (s.R.n_ranks > 1) {
+        uint32_t wn = s.wn[w];
+        warp_flush_remote<APP>(s, kp, cta, w, true, wn);
+        __syncwarp();
+        if ((tid & 31) == 0) s.wn[w] = wn;
+        __syncthreads();
+    }
+    if (tid == 0) {
+        uint32_t total = 0;
+        for (int k = 0; k < kWarps; ++k) { s.wpre[k] = total; total += s.wn[k]; }
+        s.wpre[kWarps] = total;
+        uint32_t keep_n = 0;
+        if (allow_keep && kp.keep > 0 && total > 0 && total <= (uint32_t)kp.keep) {
+            // keep only in a low-parallelism phase: the rank's whole outstanding
+            // work (T - F, this batch included) is tiny, so enqueueing would only
+            // add a queue round trip per level (path/road-like graphs); otherwise
+            // FIFO order is kept, which bounds asynchronous redundancy.
+            const uint64_t f = ld_relaxed_gpu(&s.R.ctrl->finished.v), t = ld_relaxed_gpu(&s.R.ctrl->tail.v);
+            if (t - f <= (uint64_t)kp.keep) keep_n = total;
+        }
+        const uint32_t push_n = total - keep_n;
+        s.b64[0] = push_n ? atomicAdd((unsigned long long *)&s.R.ctrl->tail.v, (unsigned long long)push_n) : 0ull;
+        s.b32[0] = (int32_t)keep_n;
+        s.b32[1] = (int32_t)total;
+        s.c_pushes += push_n;
+    }
+    __syncthreads();
+    const uint32_t keep_n = (uint32_t)s.b32[0], total = (uint32_t)s.b32[1];
+    const uint64_t base = s.b64[0];
+    if (total > keep_n) fence_acq_rel_gpu();   // release state updates before the items are visible
+    for (uint32_t i = tid; i < total; i += kThreads) {
+        int k = 0;
+        while (k + 1 < kWarps && s.wpre[k + 1] <= i) ++k;
+        const uint32_t item = s.wout[k][i - s.wpre[k]];
+        if (i < keep_n) s.v[i] = item;
+        else ring_store(s.R, base + (i - keep_n), item, s.ring_base);
+    }
+    __syncthreads();
+    if (tid < kWarps) s.wn[tid] = 0;
+    __syncthreads();
+    return (int)keep_n;
+}
+
+// Report this CTA's staged-message count change to the rank counter.
+__device__ void report_staged(Smem &s) {
+    if (s.R.n_ranks <= 1) return;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint64_t cur = 0;
+        for (int w = 0; w < kWarps; ++w)
+            for (int d = 0; d < s.R.n_ranks; ++d) cur += (uint64_t)(s.wst[w][d] - s.wsh[w][d]);
+        const uint64_t delta = cur - s.staged_reported;   // mod 2^64
+        if (delta != 0) {
+            fence_acq_rel_sys();
+            atomicAdd((unsigned long long *)&s.R.ctrl->staged.v, (unsigned long long)delta);
+            s.staged_reported = cur;
+        }
+    }
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------
+// pop from the local ring: reserve-then-wait
+// ---------------------------------------------------------------------------
+__device__ int pop_batch(Smem &s, const KParams &kp) {
+    const RankDev &R = s.R;
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        if (s.res_lo == s.res_hi) {
+            const uint64_t t = ld_relaxed_gpu(&R.ctrl->tail.v);
+            const uint64_t h = ld_relaxed_gpu(&R.ctrl->head.v);
+            if (t > h) {
+                uint64_t k = (t - h) / (uint64_t)kp.ctas_per_rank;
+                k = k < 1 ? 1 : (k > (uint64_t)kp.fetch ? (uint64_t)kp.fetch : k);
+                const uint64_t lo = atomicAdd((unsigned long long *)&R.ctrl->head.v, (unsigned long long)k);
+                s.res_lo = lo;
+                s.res_hi = lo + k;
+            }
+        }
+        s.minbad = kThreads;
+    }
+    __syncthreads();
+    const uint64_t lo = s.res_lo;
+    const uint64_t avail = s.res_hi - lo;
+    const int cnt = (int)(avail < (uint64_t)kp.fetch ? avail : (uint64_t)kp.fetch);
+    const uint64_t idx = lo + tid;
+    uint64_t slot = 0;
+    if (tid < cnt) {
+        slot = ld_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)]);
+        if (!slot_full_for(slot, idx)) atomicMin(&s.minbad, tid);
+    }
+    __syncthreads();
+    const int B = cnt < s.minbad ? cnt : s.minbad;
+    if (tid < B) {
+        fence_acq_rel_gpu();   // acquire: see the producer's state update of this vertex
+        s.v[tid] = lo32(slot);
+        st_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)], pack(lo32(idx + R.ring_cap), 0u));
+    }
+    __syncthreads();
+    if (tid == 0) s.res_lo = lo + (uint64_t)B;
+    return B;
+}
+
+// ---------------------------------------------------------------------------
+// termination (multi-rank): coordinator double wave
+// ---------------------------------------------------------------------------
+// Rank 0, CTA 0, warp 0 reads every rank's (F, R, T, staged, S); done when two
+// consecutive waves are identical, every rank is passive (F == T, staged == 0)
+// and sum S == sum R (Mattern's four-counter method).
+__device__ void coordinator_step(Smem &s, const KParams &kp) {
+    const RankDev &R = s.R;
+    if (threadIdx.x >= 32) return;
+    const int lane = threadIdx.x;
+    const int p = R.n_ranks;
+    bool started = true;
+    uint64_t F = 0, Rv = 0, T = 0, St = 0, S = 0;
+    if (lane < p) {
+        started = ld_acquire_sys(&R.ctrl->started[lane].v) == kp.epoch;
+        const Ctrl *c = R.peer_ctrl[lane];
+        F = ld_acquire_sys(&c->finished.v);
+        Rv = ld_acquire_sys(&c->recvd.v);
+        T = ld_acquire_sys(&c->tail.v);
+        St = ld_acquire_sys(&c->staged.v);
+        S = ld_acquire_sys(&c->sent.v);
+    }
+    if (!__all_sync(kFull, started)) {
+        if (lane == 0) s.wave_valid = 0;
+        __syncwarp();
+        return;
+    }
+    bool same = true, passive = true;
+    if (lane < p) {
+        same = s.wave_valid && s.wave[lane][0] == F && s.wave[lane][1] == Rv && s.wave[lane][2] == T &&
+               s.wave[lane][3] == St && s.wave[lane][4] == S;
+        passive = (F == T) && (St == 0);
+    }
+    uint64_t sumS = S, sumR = Rv;
+#pragma unroll
+    for (int d = 16; d >= 1; d >>= 1) {
+        sumS += __shfl_xor_sync(kFull, sumS, d);
+        sumR += __shfl_xor_sync(kFull, sumR, d);
+    }
+    const bool all_same = __all_sync(kFull, same);
+    const bool all_passive = __all_sync(kFull, passive);
+    __syncwarp();
+    if (lane < p) {
+        s.wave[lane][0] = F; s.wave[lane][1] = Rv; s.wave[lane][2] = T;
+        s.wave[lane][3] = St; s.wave[lane][4] = S;
+    }
+    if (lane == 0) s.wave_valid = all_passive && sumS == sumR;
+    if (all_same && all_passive && sumS == sumR) {
+        if (lane < p) st_release_sys(&R.peer_ctrl[lane]->done.v, kp.epoch);
+    }
+    if (lane == 0) atomicAdd((unsigned long long *)&R.ctrl->st_waves.v, 1ull);
+    __syncwarp();
+}
+
+// ---------------------------------------------------------------------------
+// the persistent worker
+// ---------------------------------------------------------------------------
+template <int APP>
+__global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    Smem &s = *reinterpret_cast<Smem *>(smem_raw);
+    const int lr = blockIdx.x / kp.ctas_per_rank;
+    const int cta = blockIdx.x % kp.ctas_per_rank;
+    const int tid = threadIdx.x, w = tid >> 5;
+    if (tid == 0) {
+        s.R = kp.ranks[lr];
+        s.res_lo = s.res_hi = 0;
+        s.ring_base = s.R.ctrl->ring_base.v;
+        s.staged_reported = 0;
+        s.wave_valid = 0;
+        s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = 0;
+        s.c_busy = s.c_batches = 0;
+    }
+    if (tid < kWarps) {
+        s.wn[tid] = 0;
+        for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
+    }
+    __syncthreads();
+    const bool multi = s.R.n_ranks > 1;
+    const bool coordinator = multi && s.R.rank == 0 && cta == 0;
+    if (tid == 0 && cta == 0) st_release_sys(&s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
+    const uint64_t t_start = globaltimer();
+    uint32_t idle_streak = 0;
+
+    for (;;) {
+        if (tid == 0) {
+            int f = 0;
+            if (ld_relaxed_gpu(&s.R.ctrl->done.v) == kp.epoch) f = 1;
+            if (ld_relaxed_gpu(&s.R.ctrl->error.v) != 0) f = 2;
+            s.flag = f;
+        }
+        __syncthreads();
+        if (s.flag) break;
+
+        const uint64_t t_work0 = (tid == 0) ? globaltimer() : 0;
+        bool worked = false;
+        if (multi) {
+            uint32_t wn = s.wn[w];
+            const bool got = warp_inbound<APP>(s, kp, w, wn);
+            __syncwarp();
+            if ((tid & 31) == 0) s.wn[w] = wn;
+            worked = __syncthreads_or(got);
+        }
+        if (!worked) {
+            int B = pop_batch(s, kp);
+            if (B > 0) {
+                const int B0 = B;
+                while (B > 0) {                 // work-keeping chain
+                    if (tid == 0) s.c_pops += B;
+                    process_batch<APP>(s, kp, cta, B);
+                    B = batch_end<APP>(s, kp, cta, true);
+                }
+                report_staged(s);
+                if (tid == 0) {
+                    if (multi) fence_acq_rel_sys(); else fence_acq_rel_gpu();
+                    atomicAdd((unsigned long long *)&s.R.ctrl->finished.v, (unsigned long long)B0);  // F last
+                }
+                worked = true;
+            }
+        }
+        if (worked) {
+            if (tid == 0) { s.c_busy += globaltimer() - t_work0; s.c_batches++; }
+            idle_streak = 0;
+            continue;
+        }
+
+        // ---- idle: flush aged staging, detect termination, watchdog
+        ++idle_streak;
+        if (multi) {
+            uint32_t wn = s.wn[w];
+            warp_flush_remote<APP>(s, kp, cta, w, true, wn);
+            warp_flush_local(s, w, wn);
+            if ((tid & 31) == 0) s.wn[w] = wn;
+            report_staged(s);
+        }
+        if (tid == 0) {
+            s.c_idle++;
+            if (!multi) {
+                const uint64_t F = ld_acquire_gpu(&s.R.ctrl->finished.v);
+                const uint64_t T = ld_acquire_gpu(&s.R.ctrl->tail.v);
+                if (F == T) st_release_gpu(&s.R.ctrl->done.v, kp.epoch);
+            }
+            if (kp.watchdog_ns > 0 && globaltimer() - t_start > (uint64_t)kp.watchdog_ns)
+                set_error(s.R, kErrTimeout);
+        }
+        if (coordinator) coordinator_step(s, kp);
+        if (idle_streak > 4) __nanosleep(idle_streak > 64 ? 256 : 32);
+    }
+    __syncthreads();
+    if (tid == 0) {
+        Ctrl *c = s.R.ctrl;
+        atomicAdd((unsigned long long *)&c->st_pops.v, s.c_pops);
+        atomicAdd((unsigned long long *)&c->st_edges.v, s.c_edges);
+        atomicAdd((unsigned long long *)&c->st_pushes.v, s.c_pushes);
+        atomicAdd((unsigned long long *)&c->st_msgs.v, s.c_msgs);
+        atomicAdd((unsigned long long *)&c->st_packets.v, s.c_packets);
+        atomicAdd((unsigned long long *)&c->st_idle.v, s.c_idle);
+        atomicAdd((unsigned long long *)&c->st_hub_chunks.v, s.c_hub);
+        atomicAdd((unsigned long long *)&c->st_busy_ns.v, s.c_busy);
+        atomicAdd((unsigned long long *)&c->st_batches.v, s.c_batches);
+    }
+}
+
+}  // namespace atos
