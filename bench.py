@@ -176,6 +176,8 @@ def main():
     ap.add_argument("--no-pr", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--agg", type=int, default=1)
+    ap.add_argument("--profile-range", action="store_true",
+                    help="cudaProfilerStart/Stop around the timed region (ncu --profile-from-start off)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("[bench] warmup raised to 3 (timing rule)")
@@ -219,6 +221,8 @@ def main():
     if world > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
+    if args.profile_range:
+        torch.cuda.profiler.start()
     with ClockSampler(local) as clk:
         ev0.record(stream)
         for s in seq:
@@ -229,6 +233,8 @@ def main():
             pops += st["pops"]
         ev1.record(stream)
         torch.cuda.synchronize()
+    if args.profile_range:
+        torch.cuda.profiler.stop()
     if world > 1:
         torch.distributed.barrier()
     ms_rank = ev0.elapsed_time(ev1)

@@ -7,7 +7,7 @@ import subprocess
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-LIB = os.path.join(PKG, "libatos.so")
+LIB = os.environ.get("ATOS_LIB") or os.path.join(PKG, "libatos.so")   # ATOS_LIB: experiment variants
 SOURCES = [os.path.join(CSRC, "atos.cu")]
 DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("atos_rt.cuh", "atos_worker.cuh", "atos_aux.cuh")] + \
     [os.path.join(ROOT, "include", "atos.h")]

@@ -34,6 +34,8 @@ class Config(ctypes.Structure):
         ("fetch_size", ctypes.c_int32),
         ("keep_items", ctypes.c_int32),
         ("l2_persist", ctypes.c_int32),
+        ("prefetch", ctypes.c_int32),
+        ("relax_red", ctypes.c_int32),
         ("ring_cap_factor", ctypes.c_double),
         ("agg_enabled", ctypes.c_int32),
         ("agg_batch_msgs", ctypes.c_int32),

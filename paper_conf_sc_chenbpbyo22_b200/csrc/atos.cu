@@ -57,6 +57,8 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->fetch_size = kThreads;
     cfg->keep_items = 0;
     cfg->l2_persist = 1;
+    cfg->prefetch = 1;
+    cfg->relax_red = 0;
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
     cfg->agg_batch_msgs = 256;
@@ -495,6 +497,8 @@ static KParams make_params(atos_graph *g) {
     kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
     kp.keep = g->cfg.keep_items;
+    kp.prefetch = g->cfg.prefetch;
+    kp.relax_red = g->cfg.relax_red;
     kp.n_hub_slots = 0;
     kp.hub_threshold = INT64_MAX;
     kp.hub_chunk = 0;

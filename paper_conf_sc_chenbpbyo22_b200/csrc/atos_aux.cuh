@@ -33,8 +33,9 @@ __global__ void init_bfs_kernel(KParams kp) {
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         const int64_t n = R.n;
-        for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
             R.depth[i] = kInf;
+        }
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
 }

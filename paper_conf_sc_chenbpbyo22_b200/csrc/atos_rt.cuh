@@ -22,8 +22,7 @@ constexpr uint32_t kDepthInf = 0x7FFFFFFFu;   // its depth field
 // second array.  Ordering by the word == ordering by depth for improvements:
 // atomicMin(w, dw(nd)) > dw(nd)  <=>  depth(w) > nd.
 __device__ __forceinline__ uint32_t dw_make(uint32_t d) { return (d << 1) | 1u; }
-__device__ __forceinline__ uint32_t dw_depth(uint32_t w) { return w >> 1; }
-constexpr int kThreads = 512;   // CTA worker
+__device__ __forceinline__ uint32_t dw_depth(uint32_t w) { return w >> 1; }constexpr int kThreads = 512;   // CTA worker
 constexpr int kWarps = kThreads / 32;
 
 // ---------------------------------------------------------------------------
@@ -73,6 +72,56 @@ __device__ __forceinline__ uint64_t globaltimer() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// Explicit global-space accesses.  The rank view lives in shared memory, so the
+// compiler cannot prove its pointers are global and would emit generic LD/ATOM;
+// these force LDG / ATOMG without a "memory" clobber (no forced smem reloads).
+__device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) {   // weak, L1-cacheable (probes)
+    uint32_t v;
+    asm volatile("ld.global.b32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint32_t atom_min_u32(uint32_t *p, uint32_t x) {
+    uint32_t o;
+    asm volatile("atom.global.min.u32 %0, [%1], %2;" : "=r"(o) : "l"(p), "r"(x));
+    return o;
+}
+__device__ __forceinline__ void red_min_u32(uint32_t *p, uint32_t x) {
+    asm volatile("red.global.min.u32 [%0], %1;" ::"l"(p), "r"(x));
+}
+__device__ __forceinline__ uint32_t atom_and_u32(uint32_t *p, uint32_t x) {
+    uint32_t o;
+    asm volatile("atom.global.and.b32 %0, [%1], %2;" : "=r"(o) : "l"(p), "r"(x));
+    return o;
+}
+__device__ __forceinline__ double atom_add_f64(double *p, double x) {
+    double o;
+    asm volatile("atom.global.add.f64 %0, [%1], %2;" : "=d"(o) : "l"(p), "d"(x));
+    return o;
+}
+__device__ __forceinline__ void red_add_f64(double *p, double x) {
+    asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(x));
+}
+__device__ __forceinline__ uint64_t atom_exch_u64(uint64_t *p, uint64_t x) {
+    uint64_t o;
+    asm volatile("atom.global.exch.b64 %0, [%1], %2;" : "=l"(o) : "l"(p), "l"(x));
+    return o;
+}
+__device__ __forceinline__ int64_t ldg_i64_nc(const int64_t *p) {   // read-only data (row offsets)
+    int64_t v;
+    asm volatile("ld.global.nc.b64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+
+// TMA bulk prefetch of [p, p+bytes) into L2 (sm_90+): one instruction per
+// adjacency list, so the column stream is already in L2 when the warps reach it.
+__device__ __forceinline__ void prefetch_l2_bulk(const void *p, uint64_t bytes) {
+    const uint64_t end = ((uint64_t)p + bytes + 15) & ~(uint64_t)15;
+    for (uint64_t x = (uint64_t)p & ~(uint64_t)15; x < end; x += (1u << 20)) {
+        const uint32_t c = end - x > (1u << 20) ? (1u << 20) : (uint32_t)(end - x);
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(x), "r"(c));
+    }
+}
+
 // L2-only (bypass the non-coherent L1) loads for data produced by other SMs/GPUs.
 __device__ __forceinline__ uint64_t ld_cg_u64(const uint64_t *p) { return __ldcg((const unsigned long long *)p); }
 __device__ __forceinline__ uint2 ld_cg_u2(const uint2 *p) { return __ldcg(p); }
@@ -166,6 +215,8 @@ struct KParams {
     int32_t stage_cap;       // staging capacity per (cta, warp, dst), messages (pow2)
     int32_t agg_on;
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
+    int32_t prefetch;        // TMA bulk-prefetch each popped adjacency list into L2
+    int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t n_hub_slots;     // pow2
     int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
     int64_t hub_chunk;       // edges per hub chunk

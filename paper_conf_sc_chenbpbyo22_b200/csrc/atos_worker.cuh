@@ -33,9 +33,13 @@ namespace atos {
 
 constexpr int kApBfs = 0;
 constexpr int kApPr = 1;
-constexpr int kU = 8;                // edges per lane in flight
+#ifndef ATOS_KU
+#define ATOS_KU 8
+#endif
+constexpr int kU = ATOS_KU;          // edges per lane in flight
 constexpr int kChunk = 32 * kU;      // edges per warp chunk
 constexpr int kWOut = 256;           // per-warp local staging (items)
+constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
 
 template <int APP> struct AppTraits;
@@ -52,6 +56,7 @@ struct Smem {
     uint32_t wn[kWarps];
     uint32_t wpre[kWarps + 1];
     uint32_t chunk_next;           // next unclaimed edge chunk of the batch
+    uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
     uint32_t wst[kWarps][kMaxRanks], wsh[kWarps][kMaxRanks];   // per-warp message staging tail/head
     uint64_t wt0[kWarps][kMaxRanks];                           // time staging became non-empty
     int64_t wsum[kWarps];
@@ -147,7 +152,7 @@ __device__ __forceinline__ void ring_store(const RankDev &R, uint64_t idx, uint3
 }
 
 // Whole warp: push wout[w][0..wn) with one leader atomic.
-__device__ void warp_flush_local(Smem &s, int w, uint32_t &wn) {
+__device__ void warp_flush_local(Smem &s, int w, uint32_t &wn, bool fence) {
     __syncwarp();
     const uint32_t cnt = wn;
     if (cnt == 0) return;
@@ -155,7 +160,14 @@ __device__ void warp_flush_local(Smem &s, int w, uint32_t &wn) {
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd((unsigned long long *)&s.R.ctrl->tail.v, (unsigned long long)cnt);
     base = __shfl_sync(kFull, base, 0);
-    fence_acq_rel_gpu();   // release this warp's state updates before the items become visible
+    if (fence) fence_acq_rel_gpu();   // fire-and-forget relaxations must be performed first
+    // No fence: every item was appended only after its improving atomic had
+    // returned (the append is control-dependent on the returned value), so the
+    // state update is already performed at L2, the coherence point, before this
+    // store is issued; the consumer's claiming atomic on the same word is
+    // address-dependent on the slot it reads.
+    // A gpu-scope fence here would also invalidate L1 (CCTL.IVALL) and with it
+    // the probe hits.
     for (uint32_t i = lane; i < cnt; i += 32) ring_store(s.R, base + i, s.wout[w][i], s.ring_base);
     if (lane == 0) atomicAdd(&s.c_pushes, (unsigned long long)cnt);
     wn = 0;
@@ -335,19 +347,19 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                 const uint64_t m = ld_cg_u64((const uint64_t *)pay + i);
                 ul = lo32(m);
                 const uint32_t ndw = dw_make(hi32(m));
-                pred = atomicMin(R.depth + R.v_begin + ul, ndw) > ndw;
+                pred = atom_min_u32(R.depth + R.v_begin + ul, ndw) > ndw;
             } else {
                 const uint4 m = ld_cg_u4((const uint4 *)pay + i);
                 ul = m.x;
                 const double dlt = __longlong_as_double((long long)(((uint64_t)m.w << 32) | m.z));
-                const double old = atomicAdd(R.pr_res + ul, dlt);
+                const double old = atom_add_f64(R.pr_res + ul, dlt);
                 pred = old < kp.eps && old + dlt >= kp.eps;
             }
         }
-        if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+        if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
         warp_append_local(s, w, wn, pred, ul);
     }
-    warp_flush_local(s, w, wn);             // T counts the new local work before R
+    warp_flush_local(s, w, wn, false);      // T counts the new local work before R
     if (lane == 0) {
         st_release_sys(&R.peer_free[src][slot], c + cp);   // slot free for the sender
         fence_acq_rel_sys();
@@ -364,8 +376,12 @@ template <int APP>
 __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
     const RankDev &R = s.R;
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    // register copies of the hot rank fields (s.R lives in smem)
     const int64_t vb = R.v_begin, ve = R.v_end;
     const bool multi = R.n_ranks > 1;
+    const int32_t *const col = R.col;
+    uint32_t *const depth = R.depth;
+    double *const res = R.pr_res;
     const uint64_t pol = policy_evict_first();
     const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
     int jprev = 0;
@@ -377,8 +393,14 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
         if (c >= nch) break;
         const int64_t c0 = (int64_t)c * kChunk;
         const int64_t clast = (E < c0 + kChunk ? E : c0 + kChunk) - 1;
-        const int jlo = upper_vertex(s, s.off[jprev] <= c0 ? jprev : 0, B - 1, c0);
-        const int jhi = upper_vertex(s, jlo, B - 1, clast);
+        int jlo, jhi;
+        if (c + 1 < (uint32_t)kChunkMap) {      // precomputed in process_batch
+            jlo = s.chunk_v[c];
+            jhi = c + 1 < nch ? s.chunk_v[c + 1] : B - 1;
+        } else {
+            jlo = upper_vertex(s, s.off[jprev] <= c0 ? jprev : 0, B - 1, c0);
+            jhi = upper_vertex(s, jlo, B - 1, clast);
+        }
         jprev = jlo;
         int j = jlo;
         int32_t u[kU];
@@ -393,25 +415,37 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                     ++j;
                     if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
                 }
-                u[k] = ld_stream(R.col + s.beg[j] + (e - s.off[j]), pol);
+                u[k] = ld_stream(col + s.beg[j] + (e - s.off[j]), pol);
                 vv[k] = s.val[j];
             }
         }
         if constexpr (APP == kApBfs) {
             uint32_t cur[kU];
 #pragma unroll
-            for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? R.depth[u[k]] : 0u;   // probe (stale = larger: safe)
+            for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;   // probe (stale = larger: safe)
             bool imp[kU];
+            if (kp.relax_red) {
+                // fire-and-forget relaxation: red.min, enqueue on the probe's verdict.
+                // A racing improver may make the entry redundant (skipped at pop by
+                // the pending bit); the flush fences before publishing the items.
 #pragma unroll
-            for (int k = 0; k < kU; ++k) {
-                const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
-                imp[k] = false;
-                if (u[k] >= 0 && ndw < cur[k]) imp[k] = atomicMin(R.depth + u[k], ndw) > ndw;
+                for (int k = 0; k < kU; ++k) {
+                    const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
+                    imp[k] = u[k] >= 0 && ndw < cur[k];
+                    if (imp[k]) red_min_u32(depth + u[k], ndw);
+                }
+            } else {
+#pragma unroll
+                for (int k = 0; k < kU; ++k) {
+                    const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
+                    imp[k] = false;
+                    if (u[k] >= 0 && ndw < cur[k]) imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
+                }
             }
 #pragma unroll
             for (int k = 0; k < kU; ++k) {
                 const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
-                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
                 warp_append_local(s, w, wn, loc, (uint32_t)(u[k] - vb));
                 if (multi) {
                     const bool rem = imp[k] && !loc;
@@ -428,13 +462,13 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                 cross[k] = false;
                 if (u[k] >= vb && u[k] < ve) {
                     const double dlt = __longlong_as_double((long long)vv[k]);
-                    const double old = atomicAdd(R.pr_res + (u[k] - vb), dlt);
+                    const double old = atom_add_f64(res + (u[k] - vb), dlt);
                     cross[k] = old < eps && old + dlt >= eps;        // crossing enqueue (R5)
                 }
             }
 #pragma unroll
             for (int k = 0; k < kU; ++k) {
-                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn);
+                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
                 warp_append_local(s, w, wn, cross[k], (uint32_t)(u[k] - vb));
                 if (multi) {
                     const bool rem = u[k] >= 0 && !(u[k] >= vb && u[k] < ve);
@@ -454,27 +488,33 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     int64_t deg = 0;
     if (tid < B) {
         const uint32_t v = s.v[tid];
-        const int64_t b = R.row_ptr[v], e = R.row_ptr[v + 1];
+        const int64_t b = ldg_i64_nc(R.row_ptr + v), e = ldg_i64_nc(R.row_ptr + v + 1);
         s.beg[tid] = b;
         deg = e - b;
         if constexpr (APP == kApBfs) {
             // claim the expansion of v at its current depth; stale duplicates see
             // the pending bit already cleared and are skipped
-            const uint32_t old = atomicAnd(R.depth + R.v_begin + v, ~1u);
+            const uint32_t old = atom_and_u32(R.depth + R.v_begin + v, ~1u);
             const uint32_t d = dw_depth(old);
             s.val[tid] = d;
             if (!(old & 1u) || d == kDepthInf) deg = 0;
         } else {
-            const double r = __longlong_as_double(
-                (long long)atomicExch((unsigned long long *)(R.pr_res + v), 0ull));
-            if (r != 0.0) atomicAdd(R.pr_rank + v, r);
+            const double r = __longlong_as_double((long long)atom_exch_u64((uint64_t *)(R.pr_res + v), 0ull));
+            if (r != 0.0) red_add_f64(R.pr_rank + v, r);
             if (r == 0.0 || deg == 0) deg = 0;        // dangling vertices absorb (R4)
             else s.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
         }
     }
+    if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + s.beg[tid], (uint64_t)deg * 4);
     int64_t excl;
     const int64_t E = block_exscan(s, deg, excl);
-    if (tid < B) s.off[tid] = excl;
+    if (tid < B) {
+        s.off[tid] = excl;
+        if (deg > 0) {   // chunk -> first vertex map: chunks starting inside this row
+            const int64_t cl = (excl + deg - 1) / kChunk;
+            for (int64_t c = (excl + kChunk - 1) / kChunk; c <= cl && c < kChunkMap; ++c) s.chunk_v[c] = (uint16_t)tid;
+        }
+    }
     if (tid == 0) { s.off[B] = E; s.c_edges += (unsigned long long)E; s.chunk_next = 0; }
     __syncthreads();
     if (E > 0) {
@@ -522,7 +562,8 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
     __syncthreads();
     const uint32_t keep_n = (uint32_t)s.b32[0], total = (uint32_t)s.b32[1];
     const uint64_t base = s.b64[0];
-    if (total > keep_n) fence_acq_rel_gpu();   // release state updates before the items are visible
+    // (no fence: see warp_flush_local; fire-and-forget relaxations need one)
+    if (APP == kApBfs && kp.relax_red && total > keep_n) fence_acq_rel_gpu();
     for (uint32_t i = tid; i < total; i += kThreads) {
         int k = 0;
         while (k + 1 < kWarps && s.wpre[k + 1] <= i) ++k;
@@ -587,7 +628,8 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
     __syncthreads();
     const int B = cnt < s.minbad ? cnt : s.minbad;
     if (tid < B) {
-        fence_acq_rel_gpu();   // acquire: see the producer's state update of this vertex
+        // no acquire fence: the vertex state is only accessed through L2 atomics
+        // whose address depends on this slot value (see warp_flush_local)
         s.v[tid] = lo32(slot);
         st_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)], pack(lo32(idx + R.ring_cap), 0u));
     }
@@ -710,7 +752,10 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
                 }
                 report_staged(s);
                 if (tid == 0) {
-                    if (multi) fence_acq_rel_sys(); else fence_acq_rel_gpu();
+                    // T (returned by its atomic before the slot stores) is performed
+                    // before this F update is issued; multi-rank adds a sys fence
+                    // because the coordinator reads these counters over NVLink
+                    if (multi) fence_acq_rel_sys();
                     atomicAdd((unsigned long long *)&s.R.ctrl->finished.v, (unsigned long long)B0);  // F last
                 }
                 worked = true;
@@ -727,7 +772,7 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
         if (multi) {
             uint32_t wn = s.wn[w];
             warp_flush_remote<APP>(s, kp, cta, w, true, wn);
-            warp_flush_local(s, w, wn);
+            warp_flush_local(s, w, wn, false);
             if ((tid & 31) == 0) s.wn[w] = wn;
             report_staged(s);
         }

@@ -38,6 +38,13 @@ def main():
     ap.add_argument("--graph", default="rmat24")
     ap.add_argument("--configs", default='[{}]')
     args = ap.parse_args()
+    try:
+        from cuda.bindings import runtime as cudart
+        _, p = cudart.cudaGetDeviceProperties(0)
+        print(f"persistingL2CacheMaxSize={p.persistingL2CacheMaxSize} accessPolicyMaxWindowSize="
+              f"{p.accessPolicyMaxWindowSize} l2={p.l2CacheSize}", flush=True)
+    except Exception as e:  # pragma: no cover
+        print("props unavailable:", e)
     t0 = time.time()
     if args.graph.startswith("path"):
         n = int(args.graph[4:])

@@ -129,6 +129,19 @@ def test_virtual_ranks_identical(vr, agg):
     assert (d >= 0).sum() > 1000
 
 
+@pytest.mark.parametrize("opts", [dict(relax_red=1), dict(relax_red=1, keep_items=64), dict(prefetch=0, l2_persist=0),
+                                  dict(keep_items=512, fetch_size=7), dict(relax_red=1, virtual_ranks=4)])
+def test_runtime_options_same_depths(opts):
+    """Every kernel option must reach the same fixed point (bit-exact depths)."""
+    g = inputs.rmat(15, 16, 2, symmetric=True)
+    rp, col = g.numpy()
+    for s in inputs.bfs_sources(g, 2, seed=5):
+        run_and_check(rp, col, s, **opts)
+    gg = inputs.road_grid(80, 60, seed=3)
+    rp, col = gg.numpy()
+    run_and_check(rp, col, 0, **opts)
+
+
 def test_virtual_ranks_tiny_packets_and_grid_bands():
     g = inputs.road_grid(120, 100, seed=1)
     rp, col = g.numpy()
