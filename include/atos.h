@@ -66,7 +66,8 @@ typedef struct {
                                  .L2) each popped adjacency list into L2      */
     int32_t relax_red;        /* BFS: 1 = fire-and-forget relaxation (red.min,
                                  enqueue on the probe's verdict; duplicates are
-                                 skipped at pop); 0 = atomicMin with return   */    double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
+                                 skipped at pop); 0 = atomicMin with return   */
+    double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
     int32_t agg_enabled;      /* communication aggregation on/off */
     int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */
     int64_t agg_max_age_ns;   /* flush age (the WAIT_TIME), globaltimer ns     */

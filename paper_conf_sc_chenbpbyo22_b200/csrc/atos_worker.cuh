@@ -92,9 +92,16 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
+#ifndef ATOS_COL_L1
+#define ATOS_COL_L1 0
+#endif
 __device__ __forceinline__ int32_t ld_stream(const int32_t *ptr, uint64_t pol) {
     int32_t v;
+#if ATOS_COL_L1
+    asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
+#else
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
+#endif
     return v;
 }
 
