@@ -67,6 +67,9 @@ typedef struct {
     int32_t relax_red;        /* BFS: 1 = fire-and-forget relaxation (red.min,
                                  enqueue on the probe's verdict; duplicates are
                                  skipped at pop); 0 = atomicMin with return   */
+    int32_t pipeline;         /* BFS: 1 = software-pipelined expansion (each
+                                 warp keeps two 128-edge chunks in flight),
+                                 2 = only for low-degree batches, 0 = never   */
     double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
     int32_t agg_enabled;      /* communication aggregation on/off */
     int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */

@@ -58,7 +58,8 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->keep_items = 0;
     cfg->l2_persist = 1;
     cfg->prefetch = 1;
-    cfg->relax_red = 0;
+    cfg->relax_red = 1;
+    cfg->pipeline = 2;
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
     cfg->agg_batch_msgs = 256;
@@ -173,6 +174,7 @@ struct atos_graph {
     Shape S{};
     int sms = 0, occ = 0, grid = 0;
     size_t persist_max = 0, window_max = 0;   // L2 persisting-cache limits of the device
+    size_t persist_set = (size_t)-1;          // carve-out last requested by this handle
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     LocalRank loc[kMaxRanks];
@@ -376,14 +378,8 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     g->sms = prop.multiProcessorCount;
     g->persist_max = (size_t)prop.persistingL2CacheMaxSize;
     g->window_max = (size_t)prop.accessPolicyMaxWindowSize;
-    if (cfg.l2_persist && g->persist_max > 0) {
-        size_t cur = 0;
-        cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-        if (cur < g->persist_max && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, g->persist_max) != cudaSuccess) {
-            cudaGetLastError();
-            g->persist_max = 0;   // not permitted here: run without the window
-        }
-    }
+    // (the persisting carve-out itself is sized per launch to the window, see launch_worker:
+    //  a carve-out larger than the window would only shrink the L2 left to everything else)
     if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
     int occ0 = 0, occ1 = 0;
     CU(kernel_setup<kApBfs>(occ0));
@@ -499,6 +495,7 @@ static KParams make_params(atos_graph *g) {
     kp.keep = g->cfg.keep_items;
     kp.prefetch = g->cfg.prefetch;
     kp.relax_red = g->cfg.relax_red;
+    kp.pipe = g->cfg.pipeline;
     kp.n_hub_slots = 0;
     kp.hub_threshold = INT64_MAX;
     kp.hub_chunk = 0;
@@ -527,10 +524,19 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
         void *base = APP == kApBfs ? (void *)(me.arena + me.L.depth) : (void *)(me.arena + me.L.res);
         size_t bytes = APP == kApBfs ? (size_t)g->n * 4 : (size_t)me.L.n_r * 8;
         bytes = std::min(bytes, g->window_max);
+        const size_t carve = std::min(bytes, g->persist_max);   // carve-out == window, no more
+        if (carve != g->persist_set) {
+            if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve) != cudaSuccess) {
+                cudaGetLastError();
+                g->persist_max = 0;                              // not permitted: no window from now on
+            } else {
+                g->persist_set = carve;
+            }
+        }
         at[na].id = cudaLaunchAttributeAccessPolicyWindow;
         at[na].val.accessPolicyWindow.base_ptr = base;
         at[na].val.accessPolicyWindow.num_bytes = bytes;
-        at[na].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)g->persist_max / (double)bytes);
+        at[na].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)carve / (double)bytes);
         at[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
         at[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
         ++na;

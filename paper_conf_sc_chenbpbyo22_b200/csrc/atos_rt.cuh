@@ -8,6 +8,7 @@
 // separate end/end_max/end_count counters (reading R15).
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 namespace atos {
@@ -75,9 +76,16 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // Explicit global-space accesses.  The rank view lives in shared memory, so the
 // compiler cannot prove its pointers are global and would emit generic LD/ATOM;
 // these force LDG / ATOMG without a "memory" clobber (no forced smem reloads).
-__device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) {   // weak, L1-cacheable (probes)
+#ifndef ATOS_PROBE_L1
+#define ATOS_PROBE_L1 1
+#endif
+__device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) {   // weak load (probes)
     uint32_t v;
+#if ATOS_PROBE_L1
     asm volatile("ld.global.b32 %0, [%1];" : "=r"(v) : "l"(p));
+#else
+    asm volatile("ld.global.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+#endif
     return v;
 }
 __device__ __forceinline__ uint32_t atom_min_u32(uint32_t *p, uint32_t x) {
@@ -217,6 +225,7 @@ struct KParams {
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
     int32_t prefetch;        // TMA bulk-prefetch each popped adjacency list into L2
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
+    int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)
     int32_t n_hub_slots;     // pow2
     int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
     int64_t hub_chunk;       // edges per hub chunk

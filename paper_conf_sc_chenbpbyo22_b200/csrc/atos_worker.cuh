@@ -70,6 +70,9 @@ struct Smem {
     uint64_t wave[kMaxRanks][5];   // coordinator double wave
     int32_t wave_valid;
     unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
+#ifdef ATOS_PROF
+    unsigned long long prof[10];
+#endif
 };
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -97,13 +100,22 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
 #endif
 __device__ __forceinline__ int32_t ld_stream(const int32_t *ptr, uint64_t pol) {
     int32_t v;
-#if ATOS_COL_L1
+#if ATOS_COL_L1 == 1
     asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
+#elif ATOS_COL_L1 == 2
+    v = __ldcs(ptr);
+#elif ATOS_COL_L1 == 3
+    v = __ldg(ptr);
 #else
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
 #endif
     return v;
 }
+
+#ifdef ATOS_PROF
+// phase timing (debug builds only): wait until `x` is available, then timestamp
+#define PROF_T(var, x) do { if ((x) == 0x7fffffff) __nanosleep(1); var = clock64(); } while (0)
+#endif
 
 // Block-wide exclusive scan of one int64 per thread; returns the total.
 __device__ __forceinline__ int64_t block_exscan(Smem &s, int64_t x, int64_t &excl) {
@@ -186,6 +198,29 @@ __device__ __forceinline__ void warp_append_local(Smem &s, int w, uint32_t &wn, 
     const uint32_t m = __ballot_sync(kFull, pred);
     if (pred) s.wout[w][wn + __popc(m & lanemask_lt())] = item;
     wn += __popc(m);
+}
+
+// Whole warp: append the items whose bit is set in each lane's mask (bit k ->
+// item[k]) with one warp scan per chunk instead of one ballot per row.
+template <int N>
+__device__ __forceinline__ void warp_append_mask(Smem &s, int w, uint32_t &wn, uint32_t msk, const uint32_t (&item)[N],
+                                                 bool fence) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t cnt = __popc(msk);
+    uint32_t incl = cnt;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, incl, d);
+        if (lane >= d) incl += y;
+    }
+    const uint32_t total = __shfl_sync(kFull, incl, 31);
+    if (total == 0) return;
+    if (wn + total > (uint32_t)kWOut) warp_flush_local(s, w, wn, fence);   // total <= 32*N <= kWOut
+    uint32_t pos = wn + incl - cnt;
+#pragma unroll
+    for (int k = 0; k < N; ++k)
+        if ((msk >> k) & 1u) s.wout[w][pos++] = item[k];
+    wn += total;
 }
 
 // ---------------------------------------------------------------------------
@@ -398,6 +433,9 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
         if (lane == 0) c = atomicAdd(&s.chunk_next, 1u);
         c = __shfl_sync(kFull, c, 0);
         if (c >= nch) break;
+#ifdef ATOS_PROF
+        long long pt0 = clock64(), pt1, pt2, pt3, pt4;
+#endif
         const int64_t c0 = (int64_t)c * kChunk;
         const int64_t clast = (E < c0 + kChunk ? E : c0 + kChunk) - 1;
         int jlo, jhi;
@@ -411,7 +449,8 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
         jprev = jlo;
         int j = jlo;
         int32_t u[kU];
-        uint64_t vv[kU];
+        using ValT = typename std::conditional<APP == kApBfs, uint32_t, uint64_t>::type;   // depth | delta bits
+        ValT vv[kU];
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
             const int64_t e = c0 + k * 32 + lane;
@@ -423,13 +462,27 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                     if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
                 }
                 u[k] = ld_stream(col + s.beg[j] + (e - s.off[j]), pol);
-                vv[k] = s.val[j];
+                vv[k] = (ValT)s.val[j];
             }
         }
+#ifdef ATOS_PROF
+        { int32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= u[k]; PROF_T(pt1, sk); }
+#endif
+#ifdef ATOS_DBG_COLONLY
+        // diagnostic build: stream the columns, skip relaxation (wrong results)
+        { int32_t sk = 0; for (int k = 0; k < kU; ++k) sk ^= u[k]; if (sk == 0x7fffffff) s.c_hub++;
+#ifdef ATOS_PROF
+          if (lane == 0) { atomicAdd(&s.prof[0], (unsigned long long)(pt1 - pt0)); atomicAdd(&s.prof[4], 1ull); }
+#endif
+          continue; }
+#endif
         if constexpr (APP == kApBfs) {
             uint32_t cur[kU];
 #pragma unroll
             for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;   // probe (stale = larger: safe)
+#ifdef ATOS_PROF
+            { uint32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= cur[k]; PROF_T(pt2, (int32_t)sk); }
+#endif
             bool imp[kU];
             if (kp.relax_red) {
                 // fire-and-forget relaxation: red.min, enqueue on the probe's verdict.
@@ -449,18 +502,39 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                     if (u[k] >= 0 && ndw < cur[k]) imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
                 }
             }
+#ifdef ATOS_PROF
+            { int32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= imp[k] ? 1 : 0; PROF_T(pt3, sk << 30); }
+#endif
+            if (!multi) {
+                uint32_t msk = 0, item[kU];
 #pragma unroll
-            for (int k = 0; k < kU; ++k) {
-                const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
-                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
-                warp_append_local(s, w, wn, loc, (uint32_t)(u[k] - vb));
-                if (multi) {
+                for (int k = 0; k < kU; ++k) {
+                    msk |= (imp[k] ? 1u : 0u) << k;
+                    item[k] = (uint32_t)(u[k] - vb);
+                }
+                warp_append_mask<kU>(s, w, wn, msk, item, kp.relax_red);
+            } else {
+#pragma unroll
+                for (int k = 0; k < kU; ++k) {
+                    const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
+                    if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
+                    warp_append_local(s, w, wn, loc, (uint32_t)(u[k] - vb));
                     const bool rem = imp[k] && !loc;
                     const int d = rem ? owner_of(R, u[k]) : 0;
                     warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
                                             (uint64_t)((uint32_t)vv[k] + 1u), wn);
                 }
             }
+#ifdef ATOS_PROF
+            pt4 = clock64();
+            if (lane == 0) {
+                atomicAdd(&s.prof[0], (unsigned long long)(pt1 - pt0));
+                atomicAdd(&s.prof[1], (unsigned long long)(pt2 - pt1));
+                atomicAdd(&s.prof[2], (unsigned long long)(pt3 - pt2));
+                atomicAdd(&s.prof[3], (unsigned long long)(pt4 - pt3));
+                atomicAdd(&s.prof[4], 1ull);
+            }
+#endif
         } else {
             const double eps = kp.eps;
             bool cross[kU];
@@ -473,17 +547,136 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                     cross[k] = old < eps && old + dlt >= eps;        // crossing enqueue (R5)
                 }
             }
+            if (!multi) {
+                uint32_t msk = 0, item[kU];
 #pragma unroll
-            for (int k = 0; k < kU; ++k) {
-                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
-                warp_append_local(s, w, wn, cross[k], (uint32_t)(u[k] - vb));
-                if (multi) {
+                for (int k = 0; k < kU; ++k) {
+                    msk |= (cross[k] ? 1u : 0u) << k;
+                    item[k] = (uint32_t)(u[k] - vb);
+                }
+                warp_append_mask<kU>(s, w, wn, msk, item, false);
+            } else {
+#pragma unroll
+                for (int k = 0; k < kU; ++k) {
+                    if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
+                    warp_append_local(s, w, wn, cross[k], (uint32_t)(u[k] - vb));
                     const bool rem = u[k] >= 0 && !(u[k] >= vb && u[k] < ve);
                     const int d = rem ? owner_of(R, u[k]) : 0;
-                    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u, vv[k], wn);
+                    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
+                                            (uint64_t)vv[k], wn);
                 }
             }
         }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// BFS expansion, software-pipelined: each warp keeps two 128-edge chunks in
+// flight -- the column loads of the next chunk are issued before the probes,
+// atomics and appends of the current one, so the HBM latency of the column
+// stream overlaps the L2 round trips of the relaxation.
+// ---------------------------------------------------------------------------
+constexpr int kPU = 4;                       // rows (of 32 edges) per pipelined stage
+constexpr int kPChunk = 32 * kPU;            // 128 edges
+static_assert(kChunk % kPChunk == 0, "pipelined chunks subdivide map chunks");
+
+struct PipeStage {
+    int32_t u[kPU];
+    uint32_t nd[kPU];
+};
+
+__device__ __forceinline__ void pipe_load(const Smem &s, int B, int64_t E, uint32_t nchm, uint32_t c, PipeStage &st,
+                                          const int32_t *col, uint64_t pol) {
+    const int lane = threadIdx.x & 31;
+    const int64_t c0 = (int64_t)c * kPChunk;
+    const int64_t clast = (E < c0 + kPChunk ? E : c0 + kPChunk) - 1;
+    const uint32_t m = (uint32_t)(c0 / kChunk);          // map chunk containing c0
+    int jlo, jhi;
+    if (m + 1 < (uint32_t)kChunkMap) {
+        jlo = s.chunk_v[m];                               // vertex of edge m*kChunk <= vertex of c0
+        jhi = m + 1 < nchm ? s.chunk_v[m + 1] : B - 1;
+    } else {
+        jlo = upper_vertex(s, 0, B - 1, c0);
+        jhi = upper_vertex(s, jlo, B - 1, clast);
+    }
+    int j = jlo;
+#pragma unroll
+    for (int k = 0; k < kPU; ++k) {
+        const int64_t e = c0 + k * 32 + lane;
+        st.u[k] = -1;
+        st.nd[k] = 0;
+        if (e <= clast) {
+            if (j < jhi && s.off[j + 1] <= e) {
+                ++j;
+                if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
+            }
+            st.u[k] = ld_stream(col + s.beg[j] + (e - s.off[j]), pol);
+            st.nd[k] = (uint32_t)s.val[j] + 1u;
+        }
+    }
+}
+
+template <int APP>
+__device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, const PipeStage &st, uint32_t &wn) {
+    const RankDev &R = s.R;
+    const int w = threadIdx.x >> 5;
+    const int64_t vb = R.v_begin, ve = R.v_end;
+    uint32_t *const depth = R.depth;
+    uint32_t cur[kPU];
+#pragma unroll
+    for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u32(depth + st.u[k]) : 0u;   // probe
+    bool imp[kPU];
+    if (kp.relax_red) {
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) {
+            const uint32_t ndw = dw_make(st.nd[k]);
+            imp[k] = st.u[k] >= 0 && ndw < cur[k];
+            if (imp[k]) red_min_u32(depth + st.u[k], ndw);
+        }
+    } else {
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) {
+            const uint32_t ndw = dw_make(st.nd[k]);
+            imp[k] = false;
+            if (st.u[k] >= 0 && ndw < cur[k]) imp[k] = atom_min_u32(depth + st.u[k], ndw) > ndw;
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < kPU; ++k) {
+        const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
+        if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
+        warp_append_local(s, w, wn, loc, (uint32_t)(st.u[k] - vb));
+        if (R.n_ranks > 1) {
+            const bool rem = imp[k] && !loc;
+            const int d = rem ? owner_of(R, st.u[k]) : 0;
+            warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
+                                    (uint64_t)st.nd[k], wn);
+        }
+    }
+}
+
+template <int APP>
+__device__ void expand_warp_pipe(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
+    const int lane = threadIdx.x & 31;
+    const int32_t *const col = s.R.col;
+    const uint64_t pol = policy_evict_first();
+    const uint32_t nchm = (uint32_t)((E + kChunk - 1) / kChunk);
+    const uint32_t nch = (uint32_t)((E + kPChunk - 1) / kPChunk);
+    uint32_t c = 0;
+    if (lane == 0) c = atomicAdd(&s.chunk_next, 1u);
+    c = __shfl_sync(kFull, c, 0);
+    if (c >= nch) return;
+    PipeStage a, b;
+    pipe_load(s, B, E, nchm, c, a, col, pol);
+    for (;;) {
+        uint32_t c2 = 0;
+        if (lane == 0) c2 = atomicAdd(&s.chunk_next, 1u);
+        c2 = __shfl_sync(kFull, c2, 0);
+        const bool more = c2 < nch;
+        if (more) pipe_load(s, B, E, nchm, c2, b, col, pol);   // next chunk's columns in flight
+        pipe_relax<APP>(s, kp, cta, a, wn);
+        if (!more) break;
+        a = b;
     }
 }
 
@@ -492,6 +685,9 @@ template <int APP>
 __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x;
+#ifdef ATOS_PROF
+    if (tid == 0) s.prof[7] -= (unsigned long long)clock64();
+#endif
     int64_t deg = 0;
     if (tid < B) {
         const uint32_t v = s.v[tid];
@@ -524,10 +720,16 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     }
     if (tid == 0) { s.off[B] = E; s.c_edges += (unsigned long long)E; s.chunk_next = 0; }
     __syncthreads();
+#ifdef ATOS_PROF
+    if (tid == 0) s.prof[7] += (unsigned long long)clock64();   // minus entry below: setup+scan
+#endif
     if (E > 0) {
         const int w = tid >> 5;
         uint32_t wn = s.wn[w];
-        expand_warp<APP>(s, kp, cta, B, E, wn);
+        // pipelined expansion pays off on low-degree (latency-bound, road-like) batches
+        if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
+            expand_warp_pipe<APP>(s, kp, cta, B, E, wn);
+        else expand_warp<APP>(s, kp, cta, B, E, wn);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
@@ -717,6 +919,9 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
         s.wave_valid = 0;
         s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = 0;
         s.c_busy = s.c_batches = 0;
+#ifdef ATOS_PROF
+        for (int k = 0; k < 10; ++k) s.prof[k] = 0;
+#endif
     }
     if (tid < kWarps) {
         s.wn[tid] = 0;
@@ -749,15 +954,34 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
             worked = __syncthreads_or(got);
         }
         if (!worked) {
+#ifdef ATOS_PROF
+            const long long pb0 = clock64();
+#endif
             int B = pop_batch(s, kp);
+#ifdef ATOS_PROF
+            if (tid == 0 && B > 0) s.prof[6] += (unsigned long long)(clock64() - pb0);
+#endif
             if (B > 0) {
                 const int B0 = B;
                 while (B > 0) {                 // work-keeping chain
                     if (tid == 0) s.c_pops += B;
+#ifdef ATOS_PROF
+                    const long long pb1 = clock64();
+#endif
                     process_batch<APP>(s, kp, cta, B);
+#ifdef ATOS_PROF
+                    const long long pb2 = clock64();
+                    if (tid == 0) s.prof[8] += (unsigned long long)(pb2 - pb1);
+#endif
                     B = batch_end<APP>(s, kp, cta, true);
+#ifdef ATOS_PROF
+                    if (tid == 0) s.prof[9] += (unsigned long long)(clock64() - pb2);
+#endif
                 }
                 report_staged(s);
+#ifdef ATOS_PROF
+                if (tid == 0) { s.prof[5] += (unsigned long long)(clock64() - pb0); }
+#endif
                 if (tid == 0) {
                     // T (returned by its atomic before the slot stores) is performed
                     // before this F update is issued; multi-rank adds a sys fence
@@ -808,6 +1032,14 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
         atomicAdd((unsigned long long *)&c->st_hub_chunks.v, s.c_hub);
         atomicAdd((unsigned long long *)&c->st_busy_ns.v, s.c_busy);
         atomicAdd((unsigned long long *)&c->st_batches.v, s.c_batches);
+#ifdef ATOS_PROF
+        if (blockIdx.x < 4)
+            printf("PROF cta %d chunks %llu col %llu probe %llu atom %llu append %llu (cyc/chunk/warp) | per batch: pop %llu setup %llu expand(t0) %llu end %llu total %llu batches %llu\n",
+                   blockIdx.x, s.prof[4], s.prof[0] / (s.prof[4] + 1), s.prof[1] / (s.prof[4] + 1),
+                   s.prof[2] / (s.prof[4] + 1), s.prof[3] / (s.prof[4] + 1), s.prof[6] / (s.c_batches + 1),
+                   s.prof[7] / (s.c_batches + 1), s.prof[8] / (s.c_batches + 1), s.prof[9] / (s.c_batches + 1),
+                   s.prof[5] / (s.c_batches + 1), s.c_batches);
+#endif
     }
 }
 

@@ -37,13 +37,14 @@ __global__ void probe_k(const uint32_t *__restrict__ a, uint64_t mask, uint64_t 
 // BFS-shaped: stream 8 column entries per lane (coalesced rows), probe the
 // state word they name (random), like one chunk of the worker's edge loop.
 __global__ void chain_k(const uint32_t *__restrict__ colv, uint64_t ncol, const uint32_t *a, uint64_t iters,
-                        uint32_t *out) {
+                        uint32_t *out, int rnd = 0) {
     const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     const int lane = threadIdx.x & 31;
     uint32_t acc = 0;
     for (uint64_t it = 0; it < iters; ++it) {
-        const uint64_t base = ((it * nwarps + warp) * 256) % (ncol - 256);
+        uint64_t base = ((it * nwarps + warp) * 256) % (ncol - 256);
+        if (rnd) base = (mix(it * nwarps + warp) % (ncol / 256 - 1)) * 256;   // random 1 KB segment
         uint32_t u[8], c[8];
 #pragma unroll
         for (int k = 0; k < 8; ++k) u[k] = __ldcs(colv + base + k * 32 + lane);
@@ -51,6 +52,23 @@ __global__ void chain_k(const uint32_t *__restrict__ colv, uint64_t ncol, const 
         for (int k = 0; k < 8; ++k) c[k] = a[u[k]];
 #pragma unroll
         for (int k = 0; k < 8; ++k) acc += c[k];
+    }
+    if (acc == 0xdeadbeef) *out = acc;
+}
+
+// Random 128-byte rows (one warp-wide coalesced 4-B load each) over an array of
+// `n` u32: the shape of reading random adjacency-list segments.  8 rows per lane
+// group in flight.  Measures rows/s; comparing array sizes exposes TLB reach.
+__global__ void rows_k(const uint32_t *__restrict__ a, uint64_t nrows, uint64_t iters, uint32_t *out) {
+    const int lane = threadIdx.x & 31;
+    uint64_t s = mix(((blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5) * 7919ull + 17);
+    uint32_t acc = 0;
+    for (uint64_t it = 0; it < iters; ++it) {
+        uint32_t v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) { s = mix(s + k); v[k] = __ldcs(a + (s & (nrows - 1)) * 32 + lane); }
+#pragma unroll
+        for (int k = 0; k < 8; ++k) acc += v[k];
     }
     if (acc == 0xdeadbeef) *out = acc;
 }
@@ -148,7 +166,26 @@ int main() {
         cudaEventRecord(e0); chain_k<<<g4, 512>>>(colv, ncol, a, it2, out); cudaEventRecord(e1);
         cudaEventSynchronize(e1); cudaEventElapsedTime(&ms, e0, e1);
         printf(", \"chain_col_probe_occ4x512_gedges\": %.1f", (double)g4 * 512 / 32 * 256 * it2 / (ms * 1e-3) / 1e9);
+        cudaEventRecord(e0); chain_k<<<g2, 512>>>(colv, ncol, a, it2, out, 1); cudaEventRecord(e1);
+        cudaEventSynchronize(e1); cudaEventElapsedTime(&ms, e0, e1);
+        printf(", \"chain_randseg_probe_occ2x512_gedges\": %.1f", (double)g2 * 512 / 32 * 256 * it2 / (ms * 1e-3) / 1e9);
         cudaFree(colv);
+        cudaFree(a);
+    }
+    // 2c. random 128-B rows over 64 MB .. 4 GB (adjacency-segment reads; TLB reach)
+    {
+        const size_t maxb = (size_t)4 << 30;
+        uint32_t *a; CK(cudaMalloc(&a, maxb)); CK(cudaMemset(a, 0, maxb));
+        const int g2 = p.multiProcessorCount * 2;
+        for (size_t mb : {64, 256, 512, 1024, 2048, 4096}) {
+            const uint64_t nrows = (mb << 20) / 128;
+            const uint64_t iters = 64;
+            rows_k<<<g2, 512>>>(a, nrows, 4, out);
+            cudaEventRecord(e0); rows_k<<<g2, 512>>>(a, nrows, iters, out); cudaEventRecord(e1);
+            cudaEventSynchronize(e1); cudaEventElapsedTime(&ms, e0, e1);
+            const double rows = (double)g2 * 512 / 32 * 8 * iters;
+            printf(", \"rows128_%zuMB_grows\": %.2f", mb, rows / (ms * 1e-3) / 1e9);
+        }
         cudaFree(a);
     }
     // 3. random fp64 atomicAdd with return into 8 MB (RMAT-20 residuals) and 64 MB
