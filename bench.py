@@ -41,8 +41,20 @@ WORKLOADS = {
     "bfs_rmat26": ("rmat26", "bfs"),
     "bfs_kron12": ("kron12", "bfs"),
     "bfs_grid4900": ("grid4900", "bfs"),
+    "bfs_rmat18": ("rmat18", "bfs"),      # quick-check size (not a BASELINE config)
 }
 KERNELS_PER_BFS_STEP = {1: 5}    # init, seed, worker, fixup, gather (+ barrier when N > 1)
+
+
+METRIC = "BFS & PageRank GTEPS (max over ranks); headline = BFS GTEPS"
+
+
+def arm_config(args, g, srcs, world):
+    """The `config` object both arms report (same workload, same keys)."""
+    return {"workload": args.workload, "graph": g.name, "n": g.n, "nnz": g.nnz,
+            "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
+            "aggregation": bool(args.agg),
+            "l2": "no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9)}
 
 
 def log(*a):
@@ -151,12 +163,11 @@ def run_reference(args, rank, world):
         edges += int(deg[d >= 0].sum())
     dt = time.perf_counter() - t0
     v = edges / dt / 1e9
-    line = {"impl": "reference", "metric": "BFS GTEPS (RMAT, 1-D partition) -- CPU oracle",
+    line = {"impl": "reference", "metric": METRIC,
             "value": v, "unit": "GTEPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True, "scaling": "strong",
-            "vs_baseline": None, "dtype": "i32", "data": "synthetic",
-            "config": {"workload": f"{args.workload}", "graph": g.name, "n": g.n, "nnz": g.nnz,
-                       "sources": len(srcs)},
+            "vs_baseline": None, "dtype": "i32", "data": "synthetic (seeded Graph500 RMAT)",
+            "config": arm_config(args, g, srcs, world),
             "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                              "sample": f"{args.steps} serial FIFO BFS solves (oracle/oracle.c) on the full graph"},
             "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -176,6 +187,7 @@ def main():
     ap.add_argument("--no-pr", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--agg", type=int, default=1)
+    ap.add_argument("--ctas-per-sm", type=int, default=0)
     ap.add_argument("--profile-range", action="store_true",
                     help="cudaProfilerStart/Stop around the timed region (ncu --profile-from-start off)")
     args = ap.parse_args()
@@ -198,6 +210,8 @@ def main():
     srcs = [0] if gname == "kron12" else inputs.bfs_sources(g, args.sources)
     stream = torch.cuda.current_stream(dev)
     cfg = dict(agg_enabled=args.agg, stream=stream.cuda_stream)
+    if args.ctas_per_sm:
+        cfg["ctas_per_sm"] = args.ctas_per_sm
     if world > 1:
         G = adist.load_distributed(g.row_ptr, g.col, g.n, **cfg)
     else:
@@ -262,14 +276,11 @@ def main():
             "bytes_model": "8*m_reached + 28*n_reached per BFS (SURVEY 8d)",
             "worker_ms_avg": avg_worker_ms, "worker_share_of_step": avg_worker_ms / (ms / len(seq))}
 
-    line = {"metric": "BFS & PageRank GTEPS (max over ranks); headline = BFS GTEPS",
+    line = {"metric": METRIC,
             "value": value, "unit": "GTEPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms / len(seq), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic (seeded Graph500 RMAT, device-generated)",
-            "config": {"workload": args.workload, "graph": g.name, "n": g.n, "nnz": g.nnz,
-                       "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
-                       "aggregation": bool(args.agg),
-                       "l2": "no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9)},
+            "config": arm_config(args, g, srcs, world),
             "gpu_launches": args.steps * (KERNELS_PER_BFS_STEP[1] + (1 if world > 1 else 0)),
             "roofline": roof,
             "counters": {"pops_per_reached": pops / max(1, n_total), "edges_per_m_reached": edges_scanned / max(1, m_total)}}

@@ -70,6 +70,9 @@ typedef struct {
     int32_t pipeline;         /* BFS: 1 = software-pipelined expansion (each
                                  warp keeps two 128-edge chunks in flight),
                                  2 = only for low-degree batches, 0 = never   */
+    int32_t probe_filter;     /* BFS: 1 = probe a 1-byte-per-vertex depth upper
+                                 bound instead of the 4-byte words, 0 = never,
+                                 2 = when the words exceed the L2 carve-out   */
     double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
     int32_t agg_enabled;      /* communication aggregation on/off */
     int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */

@@ -37,6 +37,7 @@ class Config(ctypes.Structure):
         ("prefetch", ctypes.c_int32),
         ("relax_red", ctypes.c_int32),
         ("pipeline", ctypes.c_int32),
+        ("probe_filter", ctypes.c_int32),
         ("ring_cap_factor", ctypes.c_double),
         ("agg_enabled", ctypes.c_int32),
         ("agg_batch_msgs", ctypes.c_int32),

@@ -60,6 +60,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->prefetch = 1;
     cfg->relax_red = 1;
     cfg->pipeline = 2;
+    cfg->probe_filter = 2;
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
     cfg->agg_batch_msgs = 256;
@@ -108,7 +109,7 @@ static bool valid_cfg(const atos_config &c) {
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, total;
+    size_t ctrl, depth, filt, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -135,6 +136,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     size_t o = 0;
     L.ctrl = o;    o = al(o + sizeof(Ctrl));
     L.depth = o;   o = al(o + (size_t)S.n * 4);
+    L.filt = o;    o = al(o + (size_t)S.n);
     L.rank = o;    o = al(o + (size_t)L.n_r * 8);
     L.res = o;     o = al(o + (size_t)L.n_r * 8);
     L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
@@ -214,6 +216,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     unsigned char *b = me.arena;
     const Layout &L = me.L;
     d.depth = (uint32_t *)(b + L.depth);
+    d.filt = (uint8_t *)(b + L.filt);
     d.pr_rank = (double *)(b + L.rank);
     d.pr_res = (double *)(b + L.res);
     d.ring = (uint64_t *)(b + L.ring);
@@ -496,6 +499,10 @@ static KParams make_params(atos_graph *g) {
     kp.prefetch = g->cfg.prefetch;
     kp.relax_red = g->cfg.relax_red;
     kp.pipe = g->cfg.pipeline;
+    // probe filter: explicit, or automatically when the depth words do not fit the
+    // L2 persisting carve-out (RMAT-26: 268 MB of words, 67 MB of filter)
+    kp.filter = g->cfg.probe_filter == 1 ||
+                (g->cfg.probe_filter == 2 && (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20));
     kp.n_hub_slots = 0;
     kp.hub_threshold = INT64_MAX;
     kp.hub_chunk = 0;
@@ -521,8 +528,9 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
         // keep the random-access state (BFS words / PR residuals) resident in L2
         // while the CSR column stream passes through
         const LocalRank &me = g->loc[0];
-        void *base = APP == kApBfs ? (void *)(me.arena + me.L.depth) : (void *)(me.arena + me.L.res);
-        size_t bytes = APP == kApBfs ? (size_t)g->n * 4 : (size_t)me.L.n_r * 8;
+        void *base = APP == kApBfs ? (void *)(me.arena + (kp.filter ? me.L.filt : me.L.depth))
+                                   : (void *)(me.arena + me.L.res);
+        size_t bytes = APP == kApBfs ? (size_t)g->n * (kp.filter ? 1 : 4) : (size_t)me.L.n_r * 8;
         bytes = std::min(bytes, g->window_max);
         const size_t carve = std::min(bytes, g->persist_max);   // carve-out == window, no more
         if (carve != g->persist_set) {

@@ -35,6 +35,7 @@ __global__ void init_bfs_kernel(KParams kp) {
         const int64_t n = R.n;
         for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
             R.depth[i] = kInf;
+            R.filt[i] = 255;
         }
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
@@ -48,6 +49,7 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
         R.ctrl->ring_base.v = R.ctrl->tail.v;
         if (src < R.v_begin || src >= R.v_end) continue;
         R.depth[src] = dw_make(0);
+        R.filt[src] = 0;
         const uint64_t idx = R.ctrl->tail.v;
         uint64_t *p = &R.ring[idx & (R.ring_cap - 1)];
         if (!slot_free_for(*p, idx)) { R.ctrl->error.v = kErrCapacity; return; }

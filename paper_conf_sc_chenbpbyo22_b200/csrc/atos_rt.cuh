@@ -23,7 +23,24 @@ constexpr uint32_t kDepthInf = 0x7FFFFFFFu;   // its depth field
 // second array.  Ordering by the word == ordering by depth for improvements:
 // atomicMin(w, dw(nd)) > dw(nd)  <=>  depth(w) > nd.
 __device__ __forceinline__ uint32_t dw_make(uint32_t d) { return (d << 1) | 1u; }
-__device__ __forceinline__ uint32_t dw_depth(uint32_t w) { return w >> 1; }constexpr int kThreads = 512;   // CTA worker
+__device__ __forceinline__ uint32_t dw_depth(uint32_t w) { return w >> 1; }
+
+// BFS probe filter (used when the depth words do not fit the L2 carve-out, e.g.
+// RMAT-26: 268 MB of words vs 67 MB of filter): one byte per vertex holding an
+// upper bound of its depth, saturated at 255.  It is written after every
+// improvement with the new candidate depth; racing stores can only leave a larger
+// value, never one below the true depth, so filt[u] <= nd (unsaturated) proves the
+// edge cannot improve u.
+__device__ __forceinline__ uint8_t filt_of(uint32_t d) { return d < 255u ? (uint8_t)d : (uint8_t)255; }
+__device__ __forceinline__ bool filt_maybe(uint32_t f, uint32_t nd) { return nd < f || f == 255u; }
+__device__ __forceinline__ uint32_t ldg_u8(const uint8_t *p) {
+    uint16_t v;
+    asm volatile("ld.global.u8 %0, [%1];" : "=h"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ void stg_u8(uint8_t *p, uint32_t x) {
+    asm volatile("st.global.u8 [%0], %1;" ::"l"(p), "h"((uint16_t)x));
+}constexpr int kThreads = 512;   // CTA worker
 constexpr int kWarps = kThreads / 32;
 
 // ---------------------------------------------------------------------------
@@ -189,6 +206,7 @@ struct RankDev {
     const int32_t *col;          // [m_r] global vertex ids
     // application state (own memory)
     uint32_t *depth;             // BFS: [n] global-indexed words dw (owned + ghost filter)
+    uint8_t *filt;               // BFS: [n] probe filter, an upper bound of depth saturated at 255
     double *pr_rank;             // PR: [n_r]
     double *pr_res;              // PR: [n_r]
     // local ring (own memory)
@@ -226,6 +244,7 @@ struct KParams {
     int32_t prefetch;        // TMA bulk-prefetch each popped adjacency list into L2
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)
+    int32_t filter;          // BFS: probe the u8 filter instead of the depth words
     int32_t n_hub_slots;     // pow2
     int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
     int64_t hub_chunk;       // edges per hub chunk

@@ -390,6 +390,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                 ul = lo32(m);
                 const uint32_t ndw = dw_make(hi32(m));
                 pred = atom_min_u32(R.depth + R.v_begin + ul, ndw) > ndw;
+                if (pred && kp.filter) stg_u8(R.filt + R.v_begin + ul, filt_of(hi32(m)));
             } else {
                 const uint4 m = ld_cg_u4((const uint4 *)pay + i);
                 ul = m.x;
@@ -478,8 +479,15 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
 #endif
         if constexpr (APP == kApBfs) {
             uint32_t cur[kU];
+            uint8_t *const filt = R.filt;
+            const bool fl = kp.filter;
+            if (fl) {
 #pragma unroll
-            for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;   // probe (stale = larger: safe)
+                for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u8(filt + u[k]) : 0u;     // probe the filter
+            } else {
+#pragma unroll
+                for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;   // probe (stale = larger: safe)
+            }
 #ifdef ATOS_PROF
             { uint32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= cur[k]; PROF_T(pt2, (int32_t)sk); }
 #endif
@@ -490,16 +498,22 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                 // the pending bit); the flush fences before publishing the items.
 #pragma unroll
                 for (int k = 0; k < kU; ++k) {
-                    const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
-                    imp[k] = u[k] >= 0 && ndw < cur[k];
-                    if (imp[k]) red_min_u32(depth + u[k], ndw);
+                    const uint32_t nd = (uint32_t)vv[k] + 1u, ndw = dw_make(nd);
+                    imp[k] = u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k]);
+                    if (imp[k]) {
+                        red_min_u32(depth + u[k], ndw);
+                        if (fl) stg_u8(filt + u[k], filt_of(nd));
+                    }
                 }
             } else {
 #pragma unroll
                 for (int k = 0; k < kU; ++k) {
-                    const uint32_t ndw = dw_make((uint32_t)vv[k] + 1u);
+                    const uint32_t nd = (uint32_t)vv[k] + 1u, ndw = dw_make(nd);
                     imp[k] = false;
-                    if (u[k] >= 0 && ndw < cur[k]) imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
+                    if (u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k])) {
+                        imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
+                        if (fl && imp[k]) stg_u8(filt + u[k], filt_of(nd));
+                    }
                 }
             }
 #ifdef ATOS_PROF
@@ -622,23 +636,36 @@ __device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, 
     const int w = threadIdx.x >> 5;
     const int64_t vb = R.v_begin, ve = R.v_end;
     uint32_t *const depth = R.depth;
+    uint8_t *const filt = R.filt;
+    const bool fl = kp.filter;
     uint32_t cur[kPU];
+    if (fl) {
 #pragma unroll
-    for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u32(depth + st.u[k]) : 0u;   // probe
+        for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u8(filt + st.u[k]) : 0u;
+    } else {
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u32(depth + st.u[k]) : 0u;   // probe
+    }
     bool imp[kPU];
     if (kp.relax_red) {
 #pragma unroll
         for (int k = 0; k < kPU; ++k) {
             const uint32_t ndw = dw_make(st.nd[k]);
-            imp[k] = st.u[k] >= 0 && ndw < cur[k];
-            if (imp[k]) red_min_u32(depth + st.u[k], ndw);
+            imp[k] = st.u[k] >= 0 && (fl ? filt_maybe(cur[k], st.nd[k]) : ndw < cur[k]);
+            if (imp[k]) {
+                red_min_u32(depth + st.u[k], ndw);
+                if (fl) stg_u8(filt + st.u[k], filt_of(st.nd[k]));
+            }
         }
     } else {
 #pragma unroll
         for (int k = 0; k < kPU; ++k) {
             const uint32_t ndw = dw_make(st.nd[k]);
             imp[k] = false;
-            if (st.u[k] >= 0 && ndw < cur[k]) imp[k] = atom_min_u32(depth + st.u[k], ndw) > ndw;
+            if (st.u[k] >= 0 && (fl ? filt_maybe(cur[k], st.nd[k]) : ndw < cur[k])) {
+                imp[k] = atom_min_u32(depth + st.u[k], ndw) > ndw;
+                if (fl && imp[k]) stg_u8(filt + st.u[k], filt_of(st.nd[k]));
+            }
         }
     }
 #pragma unroll

@@ -15,18 +15,24 @@ import torch.distributed as dist
 
 
 def env_rank_world():
-    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), \
-        int(os.environ.get("LOCAL_RANK", os.environ.get("RANK", "0")))
+    local = int(os.environ.get("LOCAL_RANK", os.environ.get("RANK", "0")))
+    if os.environ.get("ATOS_SAME_DEVICE"):      # test mode: every rank on device 0 (time-sliced)
+        local = 0
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), local
 
 
 def init(backend: Optional[str] = None):
-    """Initialise the default process group from torchrun env (127.0.0.1 rendezvous)."""
+    """Initialise the default process group from torchrun env (127.0.0.1 rendezvous).
+    Backend: ATOS_DIST_BACKEND, else NCCL with a GPU (gloo when ATOS_SAME_DEVICE is set,
+    since NCCL refuses two ranks on one GPU), else gloo."""
     rank, world, local = env_rank_world()
     if world > 1 and not dist.is_initialized():
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", "29533")
         if backend is None:
-            backend = "nccl" if torch.cuda.is_available() else "gloo"
+            backend = os.environ.get("ATOS_DIST_BACKEND")
+        if backend is None:
+            backend = "nccl" if torch.cuda.is_available() and not os.environ.get("ATOS_SAME_DEVICE") else "gloo"
         if backend == "nccl":
             torch.cuda.set_device(local)
         dist.init_process_group(backend, rank=rank, world_size=world)

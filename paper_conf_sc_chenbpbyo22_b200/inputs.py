@@ -249,6 +249,8 @@ CONFIGS = {
     "rmat26_pr": dict(kind="rmat", scale=26, edgefactor=16, symmetric=False, permute=True, app="pr"),
     # north_star target: BFS RMAT-26 symmetric
     "rmat26": dict(kind="rmat", scale=26, edgefactor=16, symmetric=True, permute=True, app="bfs"),
+    # quick-check size for multi-process smoke runs (not a BASELINE config)
+    "rmat18": dict(kind="rmat", scale=18, edgefactor=16, symmetric=True, permute=True, app="bfs"),
 }
 
 

@@ -84,10 +84,12 @@ def test_isolated_source_and_disconnected():
     assert run_and_check(rp, col, 2).tolist() == [-1, -1, 0, 1, 2, -1]
 
 
-def test_long_path_latency_bound():
+@pytest.mark.parametrize("filt", [0, 1])
+def test_long_path_latency_bound(filt):
+    """20 000 levels: also exercises the saturated (255) probe filter."""
     n = 20000
     rp, col = csr_of(n, [(i, i + 1) for i in range(n - 1)] + [(i + 1, i) for i in range(n - 1)])
-    d = run_and_check(rp, col, 0)
+    d = run_and_check(rp, col, 0, probe_filter=filt)
     assert d[-1] == n - 1
 
 
@@ -130,7 +132,10 @@ def test_virtual_ranks_identical(vr, agg):
 
 
 @pytest.mark.parametrize("opts", [dict(relax_red=1), dict(relax_red=1, keep_items=64), dict(prefetch=0, l2_persist=0),
-                                  dict(keep_items=512, fetch_size=7), dict(relax_red=1, virtual_ranks=4)])
+                                  dict(keep_items=512, fetch_size=7), dict(relax_red=1, virtual_ranks=4),
+                                  dict(relax_red=0), dict(pipeline=1), dict(pipeline=0),
+                                  dict(probe_filter=1), dict(probe_filter=1, relax_red=0),
+                                  dict(probe_filter=1, virtual_ranks=3), dict(probe_filter=1, pipeline=1)])
 def test_runtime_options_same_depths(opts):
     """Every kernel option must reach the same fixed point (bit-exact depths)."""
     g = inputs.rmat(15, 16, 2, symmetric=True)
