@@ -61,6 +61,15 @@ def log(*a):
     print(*a, file=sys.stderr, flush=True)
 
 
+def micro_peak(key):
+    """A denominator measured by scripts/micro.cu on this pool's B200 (committed under profiles/)."""
+    p = os.path.join(ROOT, "profiles", "r1", "micro_denominators.json")
+    try:
+        return float(json.load(open(p))[key])
+    except Exception:
+        return None
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -188,6 +197,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--agg", type=int, default=1)
     ap.add_argument("--ctas-per-sm", type=int, default=0)
+    ap.add_argument("--north-star", type=int, default=1, help="also time the RMAT-26 BFS target (N=1)")
     ap.add_argument("--profile-range", action="store_true",
                     help="cudaProfilerStart/Stop around the timed region (ncu --profile-from-start off)")
     args = ap.parse_args()
@@ -275,6 +285,13 @@ def main():
             "traffic": traffic, "kernel": "atos::worker_kernel<BFS>", "peak_source": peak_src,
             "bytes_model": "8*m_reached + 28*n_reached per BFS (SURVEY 8d)",
             "worker_ms_avg": avg_worker_ms, "worker_share_of_step": avg_worker_ms / (ms / len(seq))}
+    chain_peak = micro_peak("chain_randseg_probe_occ2x512_gedges")
+    scanned_rate = edges_scanned / len(seq) / world / (avg_worker_ms * 1e-3) / 1e9
+    roof["l2_probe_view"] = {
+        "what": "edges scanned per second vs the measured column-segment -> random-probe chain at the "
+                "worker's occupancy (scripts/micro.cu): the binding hardware rate for this method",
+        "achieved_gedges": scanned_rate, "peak_gedges": chain_peak,
+        "frac": scanned_rate / chain_peak if chain_peak else None}
 
     line = {"metric": METRIC,
             "value": value, "unit": "GTEPS", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -350,21 +367,66 @@ def main():
         p1.record(stream)
         torch.cuda.synchronize()
         p_ms = p0.elapsed_time(p1) / args.pr_steps
+        pr_worker_ms = sum(pr_worker) / len(pr_worker)
+        atom_peak = micro_peak("atomadd_f64_8MB_gops")
         line["pagerank"] = {"workload": "pr_rmat20 (configs[1]) alpha=0.85 eps=1e-9", "graph": gp.name,
                             "n": gp.n, "nnz": gp.nnz, "ms_per_solve": p_ms,
                             "gteps_relaxations": relax / args.pr_steps / (p_ms * 1e-3) / 1e9,
                             "gteps_nnz_per_solve": gp.nnz / (p_ms * 1e-3) / 1e9,
                             "relaxations_per_nnz": relax / args.pr_steps / gp.nnz,
                             "pops_per_vertex": pr_pops / args.pr_steps / gp.n,
-                            "worker_ms_avg": sum(pr_worker) / len(pr_worker), "dtype": "f64"}
+                            "worker_ms_avg": pr_worker_ms, "dtype": "f64",
+                            "roofline": {"bound": "l2_atomic", "unit": "Gatomic/s",
+                                         "achieved": relax / args.pr_steps / (pr_worker_ms * 1e-3) / 1e9,
+                                         "peak": atom_peak,
+                                         "frac": (relax / args.pr_steps / (pr_worker_ms * 1e-3) / 1e9 / atom_peak)
+                                         if atom_peak else None,
+                                         "peak_source": "measured fp64 atomicAdd-with-return to random addresses "
+                                                        "in an 8 MB array (scripts/micro.cu, profiles/r1)"}}
         P.free()
 
     # ---- CPU oracle baseline (rank 0, N = 1 only)
     if not args.no_cpu_baseline and world == 1 and rank == 0:
         s = seq[0]
         line["cpu_baseline"] = cpu_baseline_bfs(g, s, units[s][0])
-
     G.free()
+    del g, deg, depth
+
+    # ---- north_star target: BFS on RMAT-26 (symmetric) on one GPU
+    if args.north_star and world == 1 and args.workload == "bfs_rmat24":
+        torch.cuda.empty_cache()
+        g26 = make_graph("rmat26", dev)
+        G26 = atos.Graph(g26.row_ptr, g26.col, g26.n, **cfg)
+        d26 = torch.empty(g26.n, dtype=torch.int32, device=dev)
+        deg26 = g26.degrees()
+        srcs26 = inputs.bfs_sources(g26, 4)
+        u26 = {}
+        for s in srcs26:
+            G26.bfs(s, depth_out=d26)
+            G26.last_stats()
+            u26[s] = m_reached_of(d26, deg26)
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        wms, mt, nt = [], 0, 0
+        q0.record(stream)
+        for k in range(8):
+            s = srcs26[k % len(srcs26)]
+            G26.bfs(s, depth_out=d26)
+            wms.append(G26.last_stats()["ms_worker"])
+            mt += u26[s][0]
+            nt += u26[s][1]
+        q1.record(stream)
+        torch.cuda.synchronize()
+        ms26 = q0.elapsed_time(q1) / 8
+        bytes26 = (8 * mt + 28 * nt) / 8
+        w26 = sum(wms) / len(wms)
+        line["north_star_rmat26"] = {
+            "workload": "bfs_rmat26 (north_star target: RMAT-26 ef16 symmetric BFS, 1 GPU)", "graph": g26.name,
+            "n": g26.n, "nnz": g26.nnz, "gteps": mt / 8 / (ms26 * 1e-3) / 1e9, "ms_per_step": ms26,
+            "roofline": {"bound": "hbm", "achieved": bytes26 / (w26 * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                         "frac": bytes26 / (w26 * 1e-3) / 1e9 / peak, "bytes_model": "8*m_reached + 28*n_reached"},
+            "target": "frac >= 0.5 (BASELINE.json north_star)"}
+        G26.free()
     if rank == 0:
         print(json.dumps(line), flush=True)
 
