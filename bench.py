@@ -54,6 +54,7 @@ def arm_config(args, g, srcs, world):
     return {"workload": args.workload, "graph": g.name, "n": g.n, "nnz": g.nnz,
             "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
             "aggregation": bool(args.agg),
+            "vertex_order": "degree-relabeled inside rank blocks (atos_config.relabel=auto); outputs in generator ids",
             "l2": "no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9)}
 
 
@@ -349,7 +350,9 @@ def main():
     # ---- PageRank line of the metric (configs[1])
     if not args.no_pr and world == 1:
         gp = make_graph("rmat20_pr", dev)
-        P = atos.Graph(gp.row_ptr, gp.col, gp.n, **cfg)
+        # PR keeps the generator's (random) labels: degree relabeling measured 1.6x
+        # slower for push-PR on RMAT-20
+        P = atos.Graph(gp.row_ptr, gp.col, gp.n, **dict(cfg, relabel=0))
         r_out = torch.empty(gp.n, dtype=torch.float64, device=dev)
         s_out = torch.empty(gp.n, dtype=torch.float64, device=dev)
         P.pagerank(0.85, 1e-9, rank_out=r_out, residual_out=s_out)

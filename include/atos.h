@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define ATOS_ABI_VERSION 1
+#define ATOS_ABI_VERSION 2
 #define ATOS_MAX_RANKS 8          /* one NVSwitch box: 8 GPUs */
 #define ATOS_IPC_HANDLE_BYTES 64  /* == sizeof(cudaIpcMemHandle_t) */
 
@@ -87,6 +87,18 @@ typedef struct {
     int32_t device;           /* CUDA device ordinal                           */
     void *stream;             /* cudaStream_t to launch on; NULL = the library
                                  creates its own non-blocking stream           */
+    int32_t relabel;          /* internal vertex order (outputs and src always
+                                 use the caller's ids): 0 = as given, 1 = by
+                                 out-degree, descending, inside every rank block
+                                 (ties by id; the partition is unchanged),
+                                 2 = auto: 1 iff max degree >= 32 x mean degree
+                                 (skewed graphs)      */
+    int32_t hub_cache;        /* BFS: shared-memory depth-bound cache entries per
+                                 worker CTA for the first ids of every rank
+                                 block; multiple of 32
+                                 x n_ranks, <= 131072; 0 = off; -1 = auto
+                                 (currently off: the L1 already serves hub
+                                 probes; kept as a measured option)           */
 } atos_config;
 
 /* Per-solve statistics (device counters, summed over the ranks this handle
@@ -102,7 +114,8 @@ typedef struct {
     uint64_t packets_sent;    /* channel packets published                     */
     uint64_t bytes_sent;      /* payload bytes stored into peer channels       */
     uint64_t idle_polls;      /* worker iterations that found no work          */
-    uint64_t hub_chunks;      /* hub-split edge chunks processed               */
+    uint64_t hub_hits;        /* BFS edges retired by the shared-memory hub
+                                 cache without an L2 probe                    */
     uint64_t busy_ns;         /* sum over workers of time spent on work (ns)   */
     uint64_t batches;         /* work units (pop batches + packets + chunks)   */
     int32_t n_ranks;          /* ranks covered by these counters               */

@@ -49,6 +49,8 @@ class Config(ctypes.Structure):
         ("virtual_ranks", ctypes.c_int32),
         ("device", ctypes.c_int32),
         ("stream", ctypes.c_void_p),
+        ("relabel", ctypes.c_int32),
+        ("hub_cache", ctypes.c_int32),
     ]
 
 
@@ -63,7 +65,7 @@ class Stats(ctypes.Structure):
         ("packets_sent", ctypes.c_uint64),
         ("bytes_sent", ctypes.c_uint64),
         ("idle_polls", ctypes.c_uint64),
-        ("hub_chunks", ctypes.c_uint64),
+        ("hub_hits", ctypes.c_uint64),
         ("busy_ns", ctypes.c_uint64),
         ("batches", ctypes.c_uint64),
         ("n_ranks", ctypes.c_int32),

@@ -7,6 +7,8 @@
 // one solve (barrier -> init -> persistent worker -> fixup -> gather), error
 // and statistics plumbing.
 #include <cuda_runtime.h>
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
 
 #include <algorithm>
 #include <cstdarg>
@@ -72,6 +74,8 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->virtual_ranks = 1;
     cfg->device = 0;
     cfg->stream = nullptr;
+    cfg->relabel = 2;
+    cfg->hub_cache = -1;
     return ATOS_OK;
 }
 
@@ -102,7 +106,9 @@ static bool valid_cfg(const atos_config &c) {
            c.agg_max_age_ns >= 0 && pow2(c.channel_packets) && c.channel_packets <= (1 << 20) &&
            c.watchdog_ms >= 0 && c.n_ranks >= 1 && c.n_ranks <= ATOS_MAX_RANKS && c.rank >= 0 &&
            c.rank < c.n_ranks && c.virtual_ranks >= 1 && c.virtual_ranks <= ATOS_MAX_RANKS &&
-           !(c.virtual_ranks > 1 && c.n_ranks > 1) && c.ctas_per_sm >= 0 && c.device >= 0;
+           !(c.virtual_ranks > 1 && c.n_ranks > 1) && c.ctas_per_sm >= 0 && c.device >= 0 &&
+           c.relabel >= 0 && c.relabel <= 2 && c.hub_cache >= -1 && c.hub_cache <= kHubMax &&
+           (c.hub_cache <= 0 || c.hub_cache % (32 * std::max(c.n_ranks, c.virtual_ranks)) == 0);
 }
 
 // ---------------------------------------------------------------------------
@@ -184,6 +190,9 @@ struct atos_graph {
     bool peer_opened[kMaxRanks] = {false};
     RankDev *d_ranks = nullptr;
     int32_t *d_depth_full = nullptr;
+    int32_t *d_perm = nullptr;     // degree relabeling: old -> new (NULL = identity)
+    int32_t *d_inv = nullptr;      //                    new -> old
+    int hc_per_rank = 0;           // BFS hub-cache entries per rank block
     int64_t **d_accs = nullptr;
     uint64_t epoch = 0;
     cudaEvent_t ev_begin = nullptr, ev_w0 = nullptr, ev_w1 = nullptr, ev_end = nullptr;
@@ -193,12 +202,17 @@ struct atos_graph {
     bool last_valid = false;
 };
 
-template <int APP>
-static cudaError_t kernel_setup(int &occ) {
-    cudaError_t e = cudaFuncSetAttribute(worker_kernel<APP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)sizeof(Smem));
+// dynamic shared memory of the worker: Smem, plus the BFS hub cache (one nibble per entry)
+static size_t worker_smem(int app, int hc_entries) {
+    return sizeof(Smem) + (app == kApBfs ? (size_t)hc_entries / 2 : 0);
+}
+
+template <int APP, bool MULTI>
+static cudaError_t kernel_setup(int &occ, size_t smem) {
+    cudaError_t e = cudaFuncSetAttribute(worker_kernel<APP, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)worker_smem(APP, kHubMax));
     if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, worker_kernel<APP>, kThreads, sizeof(Smem));
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, worker_kernel<APP, MULTI>, kThreads, smem);
 }
 
 static RankDev build_view(const atos_graph *g, int lr) {
@@ -219,12 +233,14 @@ static RankDev build_view(const atos_graph *g, int lr) {
     d.filt = (uint8_t *)(b + L.filt);
     d.pr_rank = (double *)(b + L.rank);
     d.pr_res = (double *)(b + L.res);
+    d.pr_q = pr_q_of(L.n_r);
     d.ring = (uint64_t *)(b + L.ring);
     d.ring_cap = L.ring_cap;
     d.ctrl = (Ctrl *)(b + L.ctrl);
     const size_t cp = (size_t)g->S.cp, pkt = (size_t)g->S.pkt;
     d.staging = b + L.staging;
-    d.hubs = nullptr;
+    d.perm = g->d_perm;
+    d.inv = g->d_inv;
     for (int s = 0; s < g->p; ++s) {
         // base pointer of rank s's arena as seen from this process
         unsigned char *bs = nullptr;
@@ -270,6 +286,53 @@ __global__ void init_arena_kernel(uint64_t *ring, uint64_t cap, uint64_t *free_m
         free_m[i] = i % cp;            // packet slot i free for packet index i
 }
 
+// ---------------------------------------------------------------------------
+// degree relabeling: inside every rank block, vertices
+// are renumbered by out-degree, descending (ties by id), so that each block's
+// hubs have its smallest ids -- the BFS hub cache covers them, and the hot part
+// of the state arrays is compact in L2.  The partition itself is unchanged.
+// ---------------------------------------------------------------------------
+__global__ void degree_keys_kernel(const int64_t *rp, int64_t n, uint32_t *keys, int32_t *vals,
+                                   unsigned long long *maxdeg) {
+    unsigned long long mx = 0;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        int64_t d = rp[v + 1] - rp[v];
+        d = d < 0 ? 0 : (d > 0xFFFFFFFEll ? 0xFFFFFFFEll : d);
+        keys[v] = 0xFFFFFFFFu - (uint32_t)d;      // ascending key == descending degree
+        vals[v] = (int32_t)v;
+        mx = (unsigned long long)d > mx ? (unsigned long long)d : mx;
+    }
+    atomicMax(maxdeg, mx);
+}
+
+__global__ void invert_perm_kernel(const int32_t *inv, int64_t n, int32_t *perm) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        perm[inv[i]] = (int32_t)i;
+}
+
+// deg_new[i] = out-degree of the vertex that gets local id i (old rows rebased to the rank)
+__global__ void new_degrees_kernel(const int64_t *rp_old, const int32_t *inv, int64_t v0, int64_t nr,
+                                   int64_t *deg_new) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= nr; i += (int64_t)gridDim.x * blockDim.x) {
+        if (i == nr) { deg_new[i] = 0; continue; }
+        const int64_t l = (int64_t)inv[v0 + i] - v0;
+        deg_new[i] = rp_old[l + 1] - rp_old[l];
+    }
+}
+
+// one warp per new row: copy the old row, mapping every target through perm
+__global__ void permute_rows_kernel(const int64_t *rp_old, const int32_t *col_old, const int32_t *inv,
+                                    const int32_t *perm, int64_t v0, int64_t nr, const int64_t *rp_new,
+                                    int32_t *col_new) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < nr; i += nw) {
+        const int64_t l = (int64_t)inv[v0 + i] - v0;
+        const int64_t b = rp_old[l], d = rp_old[l + 1] - b, o = rp_new[i];
+        for (int64_t k = lane; k < d; k += 32) col_new[o + k] = perm[col_old[b + k]];
+    }
+}
+
 static bool is_device_ptr(const void *p) {
     if (!p) return false;
     cudaPointerAttributes a;
@@ -301,6 +364,8 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     }
     cudaFree(g->d_ranks);
     cudaFree(g->d_depth_full);
+    cudaFree(g->d_perm);
+    cudaFree(g->d_inv);
     cudaFree(g->d_accs);
     if (g->ev_begin) cudaEventDestroy(g->ev_begin);
     if (g->ev_w0) cudaEventDestroy(g->ev_w0);
@@ -329,6 +394,92 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
             cfg.fetch_size, cfg.ring_cap_factor};
     *bytes_out = make_layout(S, pt.data(), rank).total;
+    return ATOS_OK;
+}
+
+struct DevFrees {   // scratch device buffers of graph_load, freed on every exit path
+    std::vector<void *> p;
+    ~DevFrees() { for (void *x : p) cudaFree(x); }
+};
+
+// Compute g->d_inv / g->d_perm (all rank blocks, identically on every process).
+// relabel == 2 decides from the degree skew and may leave them NULL.
+static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool rp_dev) {
+    const int64_t n = g->n;
+    cudaStream_t st = g->stream;
+    DevFrees fr;
+    const int64_t *rpf = row_ptr;
+    if (!rp_dev) {
+        int64_t *t = nullptr;
+        CU(cudaMalloc(&t, (size_t)(n + 1) * 8));
+        fr.p.push_back(t);
+        CU(cudaMemcpyAsync(t, row_ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, st));
+        rpf = t;
+    }
+    uint32_t *k0 = nullptr, *k1 = nullptr;
+    int32_t *v0 = nullptr;
+    unsigned long long *d_max = nullptr;
+    CU(cudaMalloc(&k0, (size_t)n * 4)); fr.p.push_back(k0);
+    CU(cudaMalloc(&k1, (size_t)n * 4)); fr.p.push_back(k1);
+    CU(cudaMalloc(&v0, (size_t)n * 4)); fr.p.push_back(v0);
+    CU(cudaMalloc(&d_max, 8)); fr.p.push_back(d_max);
+    CU(cudaMemsetAsync(d_max, 0, 8, st));
+    degree_keys_kernel<<<1024, 256, 0, st>>>(rpf, n, k0, v0, d_max);
+    CU(cudaGetLastError());
+    unsigned long long mx = 0;
+    CU(cudaMemcpyAsync(&mx, d_max, 8, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    if (g->cfg.relabel == 2) {
+        const double mean = (double)g->nnz / (double)n;
+        if (!((double)mx >= 32.0 * std::max(1.0, mean))) return ATOS_OK;   // not skewed: keep the given order
+    }
+    CU(cudaMalloc(&g->d_inv, (size_t)n * 4));
+    CU(cudaMalloc(&g->d_perm, (size_t)n * 4));
+    int64_t maxlen = 0;
+    for (int r = 0; r < g->p; ++r) maxlen = std::max(maxlen, g->part[r + 1] - g->part[r]);
+    size_t tb = 0;
+    CU(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, v0, g->d_inv, (int)maxlen, 0, 32, st));
+    void *tmp = nullptr;
+    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    fr.p.push_back(tmp);
+    for (int r = 0; r < g->p; ++r) {
+        const int64_t b = g->part[r], len = g->part[r + 1] - b;
+        if (len <= 0) continue;
+        size_t t2 = tb;
+        CU(cub::DeviceRadixSort::SortPairs(tmp, t2, k0 + b, k1 + b, v0 + b, g->d_inv + b, (int)len, 0, 32, st));
+    }
+    invert_perm_kernel<<<1024, 256, 0, st>>>(g->d_inv, n, g->d_perm);
+    CU(cudaGetLastError());
+    CU(cudaStreamSynchronize(st));
+    return ATOS_OK;
+}
+
+// Replace rank lr's (validated, rebased) rows by the relabeled ones.
+static atos_status relabel_rows(atos_graph *g, LocalRank &me) {
+    cudaStream_t st = g->stream;
+    const int64_t v0 = g->part[me.rank], nr = me.L.n_r;
+    DevFrees fr;
+    int64_t *deg = nullptr, *rp_new = nullptr;
+    int32_t *col_new = nullptr;
+    CU(cudaMalloc(&deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
+    CU(cudaMalloc(&rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
+    CU(cudaMalloc(&col_new, (size_t)std::max<int64_t>(me.m_r, 1) * 4)); fr.p.push_back(col_new);
+    new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
+    size_t tb = 0;
+    CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
+    void *tmp = nullptr;
+    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    fr.p.push_back(tmp);
+    CU(cub::DeviceScan::ExclusiveSum(tmp, tb, deg, rp_new, (int64_t)(nr + 1), st));
+    permute_rows_kernel<<<2048, 256, 0, st>>>(me.row_ptr, me.col, g->d_inv, g->d_perm, v0, nr, rp_new, col_new);
+    CU(cudaGetLastError());
+    CU(cudaStreamSynchronize(st));
+    cudaFree(me.row_ptr);
+    cudaFree(me.col);
+    me.row_ptr = rp_new;
+    me.col = col_new;
+    fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)rp_new), fr.p.end());
+    fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)col_new), fr.p.end());
     return ATOS_OK;
 }
 
@@ -384,10 +535,12 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     // (the persisting carve-out itself is sized per launch to the window, see launch_worker:
     //  a carve-out larger than the window would only shrink the L2 left to everything else)
     if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
-    int occ0 = 0, occ1 = 0;
-    CU(kernel_setup<kApBfs>(occ0));
-    CU(kernel_setup<kApPr>(occ1));
-    g->occ = std::min(occ0, occ1);
+    int occ0 = 0, occ1 = 0, occ2 = 0, occ3 = 0;   // single- and multi-rank specialisations
+    CU((kernel_setup<kApBfs, false>(occ0, worker_smem(kApBfs, kHubMax))));
+    CU((kernel_setup<kApPr, false>(occ1, worker_smem(kApPr, 0))));
+    CU((kernel_setup<kApBfs, true>(occ2, worker_smem(kApBfs, kHubMax))));
+    CU((kernel_setup<kApPr, true>(occ3, worker_smem(kApPr, 0))));
+    g->occ = std::min(std::min(occ0, occ1), std::min(occ2, occ3));
     if (cfg.ctas_per_sm > 0) g->occ = std::min(g->occ, cfg.ctas_per_sm);
     if (g->occ < 1) return fail(ATOS_ERR_CUDA, "worker kernel cannot be resident (occupancy 0)");
     const int ctas_total = g->occ * g->sms;
@@ -408,6 +561,18 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     CU(cudaEventCreate(&g->ev_w1));
     CU(cudaEventCreate(&g->ev_end));
 
+    if (cfg.relabel != 0 && n > 1) {
+        atos_status rs = compute_relabel(g, row_ptr, rp_dev);
+        if (rs != ATOS_OK) return rs;
+    }
+    // hub cache: entries per rank block
+    {
+        int hc = cfg.hub_cache;
+        if (hc < 0) hc = 0;   // auto = off: measured slower than the L1 on RMAT-24/26
+        hc -= hc % (32 * g->p);
+        g->hc_per_rank = hc / g->p;
+    }
+
     unsigned long long *d_bad = nullptr;
     CU(cudaMalloc(&d_bad, sizeof(unsigned long long)));
     CU(cudaMemsetAsync(d_bad, 0, sizeof(unsigned long long), g->stream));
@@ -427,6 +592,14 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
         rebase_rows_kernel<<<256, 256, 0, g->stream>>>(me.row_ptr, nr + 1, rb[r]);
         check_rows_kernel<<<1024, 256, 0, g->stream>>>(me.row_ptr, nr, me.m_r, me.col, n, d_bad);
+        if (g->d_perm) {   // rows must be valid before they are permuted
+            unsigned long long bad0 = 0;
+            CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
+            CU(cudaStreamSynchronize(g->stream));
+            if (bad0) { cudaFree(d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: invalid row_ptr or column index"); }
+            atos_status rs = relabel_rows(g, me);
+            if (rs != ATOS_OK) { cudaFree(d_bad); return rs; }
+        }
         const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
         init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
                                                        (uint64_t *)(me.arena + me.L.free_m), nfree, g->S.cp);
@@ -503,9 +676,7 @@ static KParams make_params(atos_graph *g) {
     // L2 persisting carve-out (RMAT-26: 268 MB of words, 67 MB of filter)
     kp.filter = g->cfg.probe_filter == 1 ||
                 (g->cfg.probe_filter == 2 && (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20));
-    kp.n_hub_slots = 0;
-    kp.hub_threshold = INT64_MAX;
-    kp.hub_chunk = 0;
+    kp.hc_per_rank = g->hc_per_rank;
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;
@@ -517,7 +688,7 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
     cudaLaunchConfig_t lc{};
     lc.gridDim = dim3(g->grid);
     lc.blockDim = dim3(kThreads);
-    lc.dynamicSmemBytes = sizeof(Smem);
+    lc.dynamicSmemBytes = worker_smem(APP, kp.hc_per_rank * g->p);
     lc.stream = g->stream;
     cudaLaunchAttribute at[2];
     int na = 0;
@@ -551,7 +722,8 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
     }
     lc.attrs = at;
     lc.numAttrs = na;
-    CU(cudaLaunchKernelEx(&lc, worker_kernel<APP>, kp));
+    if (g->p > 1) CU(cudaLaunchKernelEx(&lc, worker_kernel<APP, true>, kp));
+    else CU(cudaLaunchKernelEx(&lc, worker_kernel<APP, false>, kp));
     return ATOS_OK;
 }
 
@@ -583,7 +755,7 @@ static atos_status finish_solve(atos_graph *g) {
         if (s != ATOS_OK) return s;
         if (c.error.v && !err) err = c.error.v;
         const uint64_t now[kSnap] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
-                                     c.st_packets.v, c.st_idle.v, c.st_hub_chunks.v, c.st_busy_ns.v,
+                                     c.st_packets.v, c.st_idle.v, c.st_hub_hits.v, c.st_busy_ns.v,
                                      c.st_batches.v};
         uint64_t *sn = g->loc[lr].snap;
         st.pops += now[0] - sn[0];
@@ -592,7 +764,7 @@ static atos_status finish_solve(atos_graph *g) {
         st.msgs_sent += now[3] - sn[3];
         st.packets_sent += now[4] - sn[4];
         st.idle_polls += now[5] - sn[5];
-        st.hub_chunks += now[6] - sn[6];
+        st.hub_hits += now[6] - sn[6];
         st.busy_ns += now[7] - sn[7];
         st.batches += now[8] - sn[8];
         std::memcpy(sn, now, sizeof(now));

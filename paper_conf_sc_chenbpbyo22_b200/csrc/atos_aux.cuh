@@ -44,6 +44,7 @@ __global__ void init_bfs_kernel(KParams kp) {
 // Seed: owner of src sets depth[src] = 0 and enqueues it.  One thread.
 __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    if (kp.ranks[0].perm) src = kp.ranks[0].perm[src];   // relabeling keeps every vertex in its rank block
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         R.ctrl->ring_base.v = R.ctrl->tail.v;
@@ -106,14 +107,16 @@ __global__ void fixup_kernel(KParams kp) {
     }
 }
 
-// Gather owned results of every rank into full-size outputs (peer loads over NVLink).
+// Gather owned results of every rank into full-size outputs (peer loads over NVLink),
+// indexed by the caller's (original) vertex ids.
 __global__ void gather_bfs_kernel(KParams kp, int32_t *out) {
     const RankDev &R = kp.ranks[0];
     const int64_t n = R.n;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         int o = 0;
         for (int k = 1; k < R.n_ranks; ++k) o += R.part[k] <= v ? 1 : 0;
-        const uint32_t d = dw_depth(__ldcg(R.peer_depth[o] + v));
+        const int64_t nv = R.perm ? R.perm[v] : v;
+        const uint32_t d = dw_depth(__ldcg(R.peer_depth[o] + nv));
         out[v] = d == kDepthInf ? -1 : (int32_t)d;
     }
 }
@@ -124,7 +127,7 @@ __global__ void gather_pr_kernel(KParams kp, double *rank_out, double *res_out) 
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         int o = 0;
         for (int k = 1; k < R.n_ranks; ++k) o += R.part[k] <= v ? 1 : 0;
-        const int64_t i = v - R.part[o];
+        const int64_t i = pr_slot((R.perm ? R.perm[v] : v) - R.part[o], pr_q_of(R.part[o + 1] - R.part[o]));
         if (rank_out) rank_out[v] = __ldcg(R.peer_rank[o] + i);
         if (res_out) res_out[v] = __ldcg(R.peer_res[o] + i);
     }
@@ -147,11 +150,11 @@ __global__ void parent_scan_kernel(KParams kp, const int32_t *depth_full, int64_
         const RankDev &R = kp.ranks[lr];
         const int64_t nr = R.v_end - R.v_begin;
         for (int64_t i = warp; i < nr; i += nwarps) {
-            const int64_t u = R.v_begin + i;
+            const int64_t u = R.inv ? R.inv[R.v_begin + i] : R.v_begin + i;   // original ids throughout
             const int32_t du = depth_full[u];
             if (du < 0) continue;
             for (int64_t e = R.row_ptr[i] + lane; e < R.row_ptr[i + 1]; e += 32) {
-                const int32_t v = R.col[e];
+                const int32_t v = R.inv ? R.inv[R.col[e]] : R.col[e];
                 if (depth_full[v] == du + 1) atomicMin((long long *)(parent_acc + v), (long long)u);
             }
         }

@@ -40,7 +40,12 @@ __device__ __forceinline__ uint32_t ldg_u8(const uint8_t *p) {
 }
 __device__ __forceinline__ void stg_u8(uint8_t *p, uint32_t x) {
     asm volatile("st.global.u8 [%0], %1;" ::"l"(p), "h"((uint16_t)x));
-}constexpr int kThreads = 512;   // CTA worker
+}
+
+#ifndef ATOS_THREADS
+#define ATOS_THREADS 512
+#endif
+constexpr int kThreads = ATOS_THREADS;   // CTA worker
 constexpr int kWarps = kThreads / 32;
 
 // ---------------------------------------------------------------------------
@@ -179,24 +184,12 @@ struct Ctrl {
     Line bar[kMaxRanks];         // pre-init barrier arrivals (epoch per rank)
     Line out_reserve[kMaxRanks]; // packets reserved on channel (this -> d)
     Line in_cursor[kMaxRanks];   // next packet to consume on channel (s -> this)
-    Line hub_count;              // hub board: number of slots ever claimed
     Line ring_base;              // tail at the start of the current solve
-    Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_chunks, st_waves;
+    Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_hits, st_waves;
     Line st_busy_ns, st_batches;
 };
 
 // Per-rank device view.  One per rank served by the grid (virtual ranks: many).
-struct HubSlot {                 // hub work-sharing board entry
-    uint64_t next;               // next edge offset to claim (atomicAdd)
-    uint64_t end;                // row end
-    uint64_t done_edges;         // edges completed (atomicAdd)
-    uint64_t total;              // total edges of the hub  (0 = slot free)
-    uint64_t epoch_tag;          // publication tag (solve epoch<<20 | slot round)
-    uint32_t v;                  // local vertex
-    uint32_t dval_lo, dval_hi;   // app value (depth / delta bits)
-    uint32_t pad_;
-};
-
 struct RankDev {
     int32_t rank, n_ranks;
     int64_t n;                   // global vertex count
@@ -207,8 +200,9 @@ struct RankDev {
     // application state (own memory)
     uint32_t *depth;             // BFS: [n] global-indexed words dw (owned + ghost filter)
     uint8_t *filt;               // BFS: [n] probe filter, an upper bound of depth saturated at 255
-    double *pr_rank;             // PR: [n_r]
-    double *pr_res;              // PR: [n_r]
+    double *pr_rank;             // PR: [n_r], stored at pr_slot(local id)
+    double *pr_res;              // PR: [n_r], stored at pr_slot(local id)
+    int64_t pr_q;                // PR slot spreading: n_r / 8 (0 = identity), see pr_slot
     // local ring (own memory)
     uint64_t *ring;
     uint64_t ring_cap;           // power of two
@@ -223,8 +217,10 @@ struct RankDev {
     uint64_t *peer_free[kMaxRanks];    // peer memory: s's free_mirror[rank]
     // CTA-private staging of outbound messages [cta][dst][stage_cap] (own memory)
     unsigned char *staging;
-    // hub board (own memory)
-    HubSlot *hubs;
+    // degree relabeling (graph_load); NULL = identity.
+    // Vertex ids inside the path are the NEW ids; outputs are mapped back.
+    const int32_t *perm;         // [n] old id -> new id
+    const int32_t *inv;          // [n] new id -> old id
     // peer state for the final gather
     uint32_t *peer_depth[kMaxRanks];
     double *peer_rank[kMaxRanks];
@@ -245,9 +241,7 @@ struct KParams {
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)
     int32_t filter;          // BFS: probe the u8 filter instead of the depth words
-    int32_t n_hub_slots;     // pow2
-    int64_t hub_threshold;   // degree above which a vertex is shared via the hub board
-    int64_t hub_chunk;       // edges per hub chunk
+    int32_t hc_per_rank;     // BFS hub cache: entries per rank block (0 = off)
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;
@@ -262,6 +256,15 @@ struct KParams {
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ bool slot_full_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx + 1); }
 __device__ __forceinline__ bool slot_free_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx); }
+
+// PR state placement: local id i lives at slot (i mod 8) * q + i / 8 (q = n_r / 8,
+// identity on the tail), so that ids adjacent after degree relabeling -- the
+// hubs, which receive most of the fp64 atomicAdds -- fall into different 32-B
+// sectors and L2 slices instead of serialising in one atomic unit.  A bijection.
+__host__ __device__ __forceinline__ int64_t pr_q_of(int64_t n_r) { return n_r >= 64 ? n_r / 8 : 0; }
+__device__ __forceinline__ int64_t pr_slot(int64_t i, int64_t q) {
+    return (q > 0 && i < 8 * q) ? (i & 7) * q + (i >> 3) : i;
+}
 
 __device__ __forceinline__ void set_error(const RankDev &R, uint64_t code) {
     atomicCAS((unsigned long long *)&R.ctrl->error.v, 0ull, (unsigned long long)code);

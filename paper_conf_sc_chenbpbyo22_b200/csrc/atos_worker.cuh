@@ -34,13 +34,14 @@ namespace atos {
 constexpr int kApBfs = 0;
 constexpr int kApPr = 1;
 #ifndef ATOS_KU
-#define ATOS_KU 8
+#define ATOS_KU 4
 #endif
 constexpr int kU = ATOS_KU;          // edges per lane in flight
 constexpr int kChunk = 32 * kU;      // edges per warp chunk
 constexpr int kWOut = 256;           // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
+constexpr int kHubMax = 131072;      // max hub-cache entries per CTA (64 KB of nibbles)
 
 template <int APP> struct AppTraits;
 template <> struct AppTraits<kApBfs> { static constexpr int kMsgBytes = 8; };
@@ -86,6 +87,35 @@ __device__ __forceinline__ int owner_of(const RankDev &R, int64_t u) {
 #pragma unroll
     for (int k = 1; k < kMaxRanks; ++k) r += (k < R.n_ranks && R.part[k] <= u) ? 1 : 0;
     return r;
+}
+
+// ---------------------------------------------------------------------------
+// BFS hub cache.  After degree relabeling the first
+// hc_per_rank ids of every rank block are that block's highest-degree vertices,
+// which receive most of the edge endpoints of a skewed graph.  Every CTA keeps a
+// shared-memory nibble per such vertex holding an UPPER BOUND of its depth word
+// (15 = unknown / >= 15).  Depths only decrease, so any value ever observed (a
+// probe result, or nd after this CTA's own relaxation) stays an upper bound
+// forever; racy read-modify-writes of the shared byte can only lose an update,
+// which leaves an older, still valid bound.  hub <= nd proves that relaxing the
+// edge cannot improve the vertex, so the edge is retired without touching L2:
+// a shared-memory lookup replaces the random global probe, whose L1TEX cost
+// (one wavefront per distinct line) is the binding limit of the BFS expansion.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint8_t *hub_base(Smem &s) { return reinterpret_cast<uint8_t *>(&s + 1); }
+
+__device__ __forceinline__ int hub_slot(const RankDev &R, int hpr, bool multi, int32_t u) {
+    if (!multi) return (uint32_t)u < (uint32_t)hpr ? u : -1;
+    const int o = owner_of(R, u);
+    const int64_t l = (int64_t)u - R.part[o];
+    return l < hpr ? o * hpr + (int)l : -1;
+}
+__device__ __forceinline__ uint32_t hub_get(const uint8_t *hc, int i) { return (hc[i >> 1] >> ((i & 1) * 4)) & 15u; }
+__device__ __forceinline__ void hub_put(uint8_t *hc, int i, uint32_t d) {
+    const uint32_t x = d < 15u ? d : 15u;
+    const int sh = (i & 1) * 4;
+    const uint32_t b = hc[i >> 1];
+    if (x < ((b >> sh) & 15u)) hc[i >> 1] = (uint8_t)((b & ~(15u << sh)) | (x << sh));
 }
 
 // Streaming loads of the column array: bypass L1, evict-first in L2 so that the
@@ -395,7 +425,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                 const uint4 m = ld_cg_u4((const uint4 *)pay + i);
                 ul = m.x;
                 const double dlt = __longlong_as_double((long long)(((uint64_t)m.w << 32) | m.z));
-                const double old = atom_add_f64(R.pr_res + ul, dlt);
+                const double old = atom_add_f64(R.pr_res + pr_slot(ul, R.pr_q), dlt);
                 pred = old < kp.eps && old + dlt >= kp.eps;
             }
         }
@@ -413,17 +443,91 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
 }
 
 // ---------------------------------------------------------------------------
+// BFS relaxation of N edges per lane (u[k] = target or -1, nd[k] = candidate
+// depth): hub-cache lookup, probe (a stale word is larger, never smaller, so a
+// probe can only cause a redundant atomic), relaxation, hub-cache update.
+// Retired edges come back with u[k] = -1 and imp[k] = false.  Whole warp.
+// ---------------------------------------------------------------------------
+template <int N, bool MULTI>
+__device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&u)[N],
+                                          const uint32_t (&nd)[N], bool (&imp)[N]) {
+    const RankDev &R = s.R;
+    uint32_t *const depth = R.depth;
+    uint8_t *const filt = R.filt;
+    const bool fl = kp.filter;
+    const int hpr = kp.hc_per_rank;
+    uint8_t *const hc = hub_base(s);
+    int hs[N];
+    if (hpr > 0) {
+        uint32_t hits = 0;
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            hs[k] = u[k] >= 0 ? hub_slot(R, hpr, MULTI, u[k]) : -1;
+            const uint32_t hb = hs[k] >= 0 ? hub_get(hc, hs[k]) : 15u;
+            if (hb < 15u && hb <= nd[k]) {   // cannot improve: retired in shared memory (15 = unknown)
+                u[k] = -1;
+                hs[k] = -1;
+                ++hits;
+            }
+        }
+        const uint32_t tot = __reduce_add_sync(kFull, hits);
+        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(&s.c_hub, (unsigned long long)tot);
+    }
+    uint32_t cur[N];
+    if (fl) {
+#pragma unroll
+        for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? ldg_u8(filt + u[k]) : 0u;       // probe the filter
+    } else {
+#pragma unroll
+        for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;     // probe the word
+    }
+    if (kp.relax_red) {
+        // fire-and-forget relaxation: red.min, enqueue on the probe's verdict.
+        // A racing improver may make the entry redundant (skipped at pop by the
+        // pending bit); the flush fences before publishing the items.
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            const uint32_t ndw = dw_make(nd[k]);
+            imp[k] = u[k] >= 0 && (fl ? filt_maybe(cur[k], nd[k]) : ndw < cur[k]);
+            if (imp[k]) {
+                red_min_u32(depth + u[k], ndw);
+                if (fl) stg_u8(filt + u[k], filt_of(nd[k]));
+            }
+        }
+    } else {
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            const uint32_t ndw = dw_make(nd[k]);
+            imp[k] = false;
+            if (u[k] >= 0 && (fl ? filt_maybe(cur[k], nd[k]) : ndw < cur[k])) {
+                imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
+                if (fl && imp[k]) stg_u8(filt + u[k], filt_of(nd[k]));
+            }
+        }
+    }
+    if (hpr > 0) {
+        // after the relaxation depth(u) <= nd; a probe that made it unnecessary saw a smaller bound
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            if (hs[k] >= 0) {
+                const uint32_t ob = fl ? cur[k] : dw_depth(cur[k]);
+                hub_put(hc, hs[k], ob < nd[k] ? ob : nd[k]);
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
 // batch expansion
 // ---------------------------------------------------------------------------
-template <int APP>
+template <int APP, bool MULTI>
 __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
     const RankDev &R = s.R;
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // register copies of the hot rank fields (s.R lives in smem)
     const int64_t vb = R.v_begin, ve = R.v_end;
-    const bool multi = R.n_ranks > 1;
+    constexpr bool multi = MULTI;
     const int32_t *const col = R.col;
-    uint32_t *const depth = R.depth;
     double *const res = R.pr_res;
     const uint64_t pol = policy_evict_first();
     const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
@@ -478,48 +582,16 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
           continue; }
 #endif
         if constexpr (APP == kApBfs) {
-            uint32_t cur[kU];
-            uint8_t *const filt = R.filt;
-            const bool fl = kp.filter;
-            if (fl) {
+            uint32_t nd[kU];
 #pragma unroll
-                for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u8(filt + u[k]) : 0u;     // probe the filter
-            } else {
-#pragma unroll
-                for (int k = 0; k < kU; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;   // probe (stale = larger: safe)
-            }
-#ifdef ATOS_PROF
-            { uint32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= cur[k]; PROF_T(pt2, (int32_t)sk); }
-#endif
+            for (int k = 0; k < kU; ++k) nd[k] = (uint32_t)vv[k] + 1u;
             bool imp[kU];
-            if (kp.relax_red) {
-                // fire-and-forget relaxation: red.min, enqueue on the probe's verdict.
-                // A racing improver may make the entry redundant (skipped at pop by
-                // the pending bit); the flush fences before publishing the items.
-#pragma unroll
-                for (int k = 0; k < kU; ++k) {
-                    const uint32_t nd = (uint32_t)vv[k] + 1u, ndw = dw_make(nd);
-                    imp[k] = u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k]);
-                    if (imp[k]) {
-                        red_min_u32(depth + u[k], ndw);
-                        if (fl) stg_u8(filt + u[k], filt_of(nd));
-                    }
-                }
-            } else {
-#pragma unroll
-                for (int k = 0; k < kU; ++k) {
-                    const uint32_t nd = (uint32_t)vv[k] + 1u, ndw = dw_make(nd);
-                    imp[k] = false;
-                    if (u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k])) {
-                        imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
-                        if (fl && imp[k]) stg_u8(filt + u[k], filt_of(nd));
-                    }
-                }
-            }
+            bfs_relax<kU, MULTI>(s, kp, u, nd, imp);
 #ifdef ATOS_PROF
+            pt2 = pt3 = pt1;
             { int32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= imp[k] ? 1 : 0; PROF_T(pt3, sk << 30); }
 #endif
-            if (!multi) {
+            if constexpr (!multi) {
                 uint32_t msk = 0, item[kU];
 #pragma unroll
                 for (int k = 0; k < kU; ++k) {
@@ -557,11 +629,11 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
                 cross[k] = false;
                 if (u[k] >= vb && u[k] < ve) {
                     const double dlt = __longlong_as_double((long long)vv[k]);
-                    const double old = atom_add_f64(res + (u[k] - vb), dlt);
+                    const double old = atom_add_f64(res + pr_slot(u[k] - vb, R.pr_q), dlt);
                     cross[k] = old < eps && old + dlt >= eps;        // crossing enqueue (R5)
                 }
             }
-            if (!multi) {
+            if constexpr (!multi) {
                 uint32_t msk = 0, item[kU];
 #pragma unroll
                 for (int k = 0; k < kU; ++k) {
@@ -590,7 +662,7 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
 // atomics and appends of the current one, so the HBM latency of the column
 // stream overlaps the L2 round trips of the relaxation.
 // ---------------------------------------------------------------------------
-constexpr int kPU = 4;                       // rows (of 32 edges) per pipelined stage
+constexpr int kPU = kU < 4 ? kU : 4;         // rows (of 32 edges) per pipelined stage
 constexpr int kPChunk = 32 * kPU;            // 128 edges
 static_assert(kChunk % kPChunk == 0, "pipelined chunks subdivide map chunks");
 
@@ -630,50 +702,19 @@ __device__ __forceinline__ void pipe_load(const Smem &s, int B, int64_t E, uint3
     }
 }
 
-template <int APP>
-__device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, const PipeStage &st, uint32_t &wn) {
+template <int APP, bool MULTI>
+__device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, PipeStage &st, uint32_t &wn) {
     const RankDev &R = s.R;
     const int w = threadIdx.x >> 5;
     const int64_t vb = R.v_begin, ve = R.v_end;
-    uint32_t *const depth = R.depth;
-    uint8_t *const filt = R.filt;
-    const bool fl = kp.filter;
-    uint32_t cur[kPU];
-    if (fl) {
-#pragma unroll
-        for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u8(filt + st.u[k]) : 0u;
-    } else {
-#pragma unroll
-        for (int k = 0; k < kPU; ++k) cur[k] = (st.u[k] >= 0) ? ldg_u32(depth + st.u[k]) : 0u;   // probe
-    }
     bool imp[kPU];
-    if (kp.relax_red) {
-#pragma unroll
-        for (int k = 0; k < kPU; ++k) {
-            const uint32_t ndw = dw_make(st.nd[k]);
-            imp[k] = st.u[k] >= 0 && (fl ? filt_maybe(cur[k], st.nd[k]) : ndw < cur[k]);
-            if (imp[k]) {
-                red_min_u32(depth + st.u[k], ndw);
-                if (fl) stg_u8(filt + st.u[k], filt_of(st.nd[k]));
-            }
-        }
-    } else {
-#pragma unroll
-        for (int k = 0; k < kPU; ++k) {
-            const uint32_t ndw = dw_make(st.nd[k]);
-            imp[k] = false;
-            if (st.u[k] >= 0 && (fl ? filt_maybe(cur[k], st.nd[k]) : ndw < cur[k])) {
-                imp[k] = atom_min_u32(depth + st.u[k], ndw) > ndw;
-                if (fl && imp[k]) stg_u8(filt + st.u[k], filt_of(st.nd[k]));
-            }
-        }
-    }
+    bfs_relax<kPU, MULTI>(s, kp, st.u, st.nd, imp);
 #pragma unroll
     for (int k = 0; k < kPU; ++k) {
         const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
         if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
         warp_append_local(s, w, wn, loc, (uint32_t)(st.u[k] - vb));
-        if (R.n_ranks > 1) {
+        if constexpr (MULTI) {
             const bool rem = imp[k] && !loc;
             const int d = rem ? owner_of(R, st.u[k]) : 0;
             warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
@@ -682,7 +723,7 @@ __device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, 
     }
 }
 
-template <int APP>
+template <int APP, bool MULTI>
 __device__ void expand_warp_pipe(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
     const int lane = threadIdx.x & 31;
     const int32_t *const col = s.R.col;
@@ -701,14 +742,14 @@ __device__ void expand_warp_pipe(Smem &s, const KParams &kp, int cta, int B, int
         c2 = __shfl_sync(kFull, c2, 0);
         const bool more = c2 < nch;
         if (more) pipe_load(s, B, E, nchm, c2, b, col, pol);   // next chunk's columns in flight
-        pipe_relax<APP>(s, kp, cta, a, wn);
+        pipe_relax<APP, MULTI>(s, kp, cta, a, wn);
         if (!more) break;
         a = b;
     }
 }
 
 // Load per-vertex info of the batch s.v[0..B) and expand it.
-template <int APP>
+template <int APP, bool MULTI>
 __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x;
@@ -729,8 +770,9 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
             s.val[tid] = d;
             if (!(old & 1u) || d == kDepthInf) deg = 0;
         } else {
-            const double r = __longlong_as_double((long long)atom_exch_u64((uint64_t *)(R.pr_res + v), 0ull));
-            if (r != 0.0) red_add_f64(R.pr_rank + v, r);
+            const int64_t sl = pr_slot(v, R.pr_q);
+            const double r = __longlong_as_double((long long)atom_exch_u64((uint64_t *)(R.pr_res + sl), 0ull));
+            if (r != 0.0) red_add_f64(R.pr_rank + sl, r);
             if (r == 0.0 || deg == 0) deg = 0;        // dangling vertices absorb (R4)
             else s.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
         }
@@ -755,8 +797,8 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         uint32_t wn = s.wn[w];
         // pipelined expansion pays off on low-degree (latency-bound, road-like) batches
         if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
-            expand_warp_pipe<APP>(s, kp, cta, B, E, wn);
-        else expand_warp<APP>(s, kp, cta, B, E, wn);
+            expand_warp_pipe<APP, MULTI>(s, kp, cta, B, E, wn);
+        else expand_warp<APP, MULTI>(s, kp, cta, B, E, wn);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
@@ -765,11 +807,11 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
 // End of a batch: publish remote staging per policy, then enqueue this CTA's
 // local discoveries with one leader atomic -- or keep up to kp.keep of them as
 // the next batch (returned count, already in s.v) when the ring is nearly empty.
-template <int APP>
+template <int APP, bool MULTI>
 __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
     const int tid = threadIdx.x, w = tid >> 5;
     __syncthreads();
-    if (s.R.n_ranks > 1) {
+    if constexpr (MULTI) {
         uint32_t wn = s.wn[w];
         warp_flush_remote<APP>(s, kp, cta, w, true, wn);
         __syncwarp();
@@ -931,8 +973,8 @@ __device__ void coordinator_step(Smem &s, const KParams &kp) {
 // ---------------------------------------------------------------------------
 // the persistent worker
 // ---------------------------------------------------------------------------
-template <int APP>
-__global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
+template <int APP, bool MULTI>
+__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KParams kp) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     Smem &s = *reinterpret_cast<Smem *>(smem_raw);
     const int lr = blockIdx.x / kp.ctas_per_rank;
@@ -954,8 +996,13 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
         s.wn[tid] = 0;
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
+    if (APP == kApBfs && kp.hc_per_rank > 0) {   // hub cache: every bound unknown (15)
+        uint32_t *hc = reinterpret_cast<uint32_t *>(hub_base(s));   // (dynamic smem is only 8-B aligned)
+        const int n4 = kp.hc_per_rank * kp.ranks[lr].n_ranks / 8;
+        for (int i = tid; i < n4; i += kThreads) hc[i] = kFull;
+    }
     __syncthreads();
-    const bool multi = s.R.n_ranks > 1;
+    constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
     if (tid == 0 && cta == 0) st_release_sys(&s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
     const uint64_t t_start = globaltimer();
@@ -973,7 +1020,7 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
 
         const uint64_t t_work0 = (tid == 0) ? globaltimer() : 0;
         bool worked = false;
-        if (multi) {
+        if constexpr (multi) {
             uint32_t wn = s.wn[w];
             const bool got = warp_inbound<APP>(s, kp, w, wn);
             __syncwarp();
@@ -995,12 +1042,12 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
 #ifdef ATOS_PROF
                     const long long pb1 = clock64();
 #endif
-                    process_batch<APP>(s, kp, cta, B);
+                    process_batch<APP, MULTI>(s, kp, cta, B);
 #ifdef ATOS_PROF
                     const long long pb2 = clock64();
                     if (tid == 0) s.prof[8] += (unsigned long long)(pb2 - pb1);
 #endif
-                    B = batch_end<APP>(s, kp, cta, true);
+                    B = batch_end<APP, MULTI>(s, kp, cta, true);
 #ifdef ATOS_PROF
                     if (tid == 0) s.prof[9] += (unsigned long long)(clock64() - pb2);
 #endif
@@ -1027,7 +1074,7 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
 
         // ---- idle: flush aged staging, detect termination, watchdog
         ++idle_streak;
-        if (multi) {
+        if constexpr (multi) {
             uint32_t wn = s.wn[w];
             warp_flush_remote<APP>(s, kp, cta, w, true, wn);
             warp_flush_local(s, w, wn, false);
@@ -1056,7 +1103,7 @@ __global__ void __launch_bounds__(kThreads, 2) worker_kernel(KParams kp) {
         atomicAdd((unsigned long long *)&c->st_msgs.v, s.c_msgs);
         atomicAdd((unsigned long long *)&c->st_packets.v, s.c_packets);
         atomicAdd((unsigned long long *)&c->st_idle.v, s.c_idle);
-        atomicAdd((unsigned long long *)&c->st_hub_chunks.v, s.c_hub);
+        atomicAdd((unsigned long long *)&c->st_hub_hits.v, s.c_hub);
         atomicAdd((unsigned long long *)&c->st_busy_ns.v, s.c_busy);
         atomicAdd((unsigned long long *)&c->st_batches.v, s.c_batches);
 #ifdef ATOS_PROF

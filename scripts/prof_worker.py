@@ -15,11 +15,13 @@ def main():
     ap.add_argument("--app", default="bfs", choices=["bfs", "pr"])
     ap.add_argument("--graph", default=None)
     ap.add_argument("--solves", type=int, default=1)
+    ap.add_argument("--cfg", default="{}", help="atos_config overrides (JSON)")
     args = ap.parse_args()
     name = args.graph or ("rmat24" if args.app == "bfs" else "rmat20_pr")
     g = inputs.make_config(name, device="cuda")
     stream = torch.cuda.current_stream()
-    G = atos.Graph(g.row_ptr, g.col, g.n, stream=stream.cuda_stream)
+    import json
+    G = atos.Graph(g.row_ptr, g.col, g.n, stream=stream.cuda_stream, **json.loads(args.cfg))
     if args.app == "bfs":
         srcs = [0] if name == "kron12" else inputs.bfs_sources(g, 4)
         depth = torch.empty(g.n, dtype=torch.int32, device="cuda")

@@ -179,3 +179,41 @@ def test_rmat24_config2_full_size():
             d = G.bfs(s)
             want = oracle.bfs(rpn, coln, s)
             assert np.array_equal(d, want)
+
+
+@pytest.mark.parametrize("opts", [dict(relabel=0), dict(relabel=1, hub_cache=0), dict(relabel=1),
+                                  dict(relabel=0, hub_cache=1024), dict(relabel=1, relax_red=0),
+                                  dict(relabel=1, probe_filter=1), dict(relabel=1, pipeline=1),
+                                  dict(relabel=1, pipeline=0, hub_cache=32),
+                                  dict(relabel=1, virtual_ranks=4, hub_cache=128),
+                                  dict(relabel=1, virtual_ranks=3, hub_cache=96 * 64),
+                                  dict(relabel=1, virtual_ranks=8, agg_enabled=0)])
+def test_relabel_and_hub_cache_same_depths_and_parents(opts):
+    """Degree relabeling and the shared-memory hub cache change the
+    internal order and retire edges without a probe; depths and the min-id
+    parents in the caller's ids must be unchanged."""
+    g = inputs.rmat(15, 16, 4, symmetric=True)
+    rp, col = g.numpy()
+    for s in inputs.bfs_sources(g, 2, seed=7):
+        run_and_check(rp, col, s, **opts)
+    gg = inputs.road_grid(70, 50, seed=4)
+    rp, col = gg.numpy()
+    run_and_check(rp, col, 3, **opts)
+    rng = np.random.default_rng(11)
+    n = 1500
+    edges = list(zip(rng.integers(0, n, 5000).tolist(), (rng.integers(0, n, 5000) // 7).tolist()))
+    rp, col = csr_of(n, edges)        # skewed in-degree, dangling rows, duplicates
+    run_and_check(rp, col, int(edges[0][0]), **opts)
+
+
+def test_hub_cache_active_on_skewed_graph():
+    g = inputs.rmat(16, 16, 1, symmetric=True)
+    rp, col = g.numpy()
+    src = inputs.bfs_sources(g, 1)[0]
+    with atos.Graph(rp, col, relabel=1, hub_cache=131072) as G:
+        d, st = G.bfs(src, stats=True)
+    assert np.array_equal(d, oracle.bfs(rp, col, src))
+    assert st["hub_hits"] > 0.2 * st["edges"], st
+    with atos.Graph(rp, col, hub_cache=0) as G:
+        d, st = G.bfs(src, stats=True)
+    assert np.array_equal(d, oracle.bfs(rp, col, src)) and st["hub_hits"] == 0

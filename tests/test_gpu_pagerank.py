@@ -110,3 +110,12 @@ def test_rmat20_config1_full_size():
     g = inputs.make_config("rmat20_pr", device="cuda")
     rp, col = g.numpy()
     run_and_check(g.row_ptr, g.col)
+
+
+@pytest.mark.parametrize("opts", [dict(relabel=0), dict(relabel=1), dict(relabel=1, virtual_ranks=4),
+                                  dict(relabel=1, virtual_ranks=3, agg_enabled=0)])
+def test_relabel_same_pagerank(opts):
+    """Outputs are in the caller's ids whatever the internal order."""
+    g = inputs.rmat(13, 16, 5, symmetric=False)
+    rp, col = g.numpy()
+    run_and_check(rp, col, **opts)
