@@ -96,7 +96,7 @@ typedef struct {
     int32_t hub_cache;        /* BFS: shared-memory depth-bound cache entries per
                                  worker CTA for the first ids of every rank
                                  block; multiple of 32
-                                 x n_ranks, <= 131072; 0 = off; -1 = auto
+                                 x n_ranks, <= 65536; 0 = off; -1 = auto
                                  (currently off: the L1 already serves hub
                                  probes; kept as a measured option)           */
 } atos_config;

@@ -59,7 +59,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->fetch_size = kThreads;
     cfg->keep_items = 0;
     cfg->l2_persist = 1;
-    cfg->prefetch = 1;
+    cfg->prefetch = 0;    // measured slower on RMAT-24 with both worker modes
     cfg->relax_red = 1;
     cfg->pipeline = 2;
     cfg->probe_filter = 2;
@@ -207,10 +207,18 @@ static size_t worker_smem(int app, int hc_entries) {
     return sizeof(Smem) + (app == kApBfs ? (size_t)hc_entries / 2 : 0);
 }
 
+// Dynamic smem limit, then the smallest shared-memory carve-out that still holds
+// `want` CTAs per SM: the rest of the 256 KB unified L1/smem stays L1, which caches
+// the hot (relabeled) part of the BFS depth words -- measured to matter.
 template <int APP, bool MULTI>
-static cudaError_t kernel_setup(int &occ, size_t smem) {
+static cudaError_t kernel_setup(int &occ, size_t smem, int want) {
     cudaError_t e = cudaFuncSetAttribute(worker_kernel<APP, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)worker_smem(APP, kHubMax));
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+    const double need_kb = (double)want * ((double)(smem + 1024 + 1024) / 1024.0);   // + static + reserved
+    int pct = (int)(need_kb / 228.0 * 100.0) + 1;
+    pct = pct > 100 ? 100 : pct;
+    e = cudaFuncSetAttribute(worker_kernel<APP, MULTI>, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
     if (e != cudaSuccess) return e;
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, worker_kernel<APP, MULTI>, kThreads, smem);
 }
@@ -535,11 +543,20 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     // (the persisting carve-out itself is sized per launch to the window, see launch_worker:
     //  a carve-out larger than the window would only shrink the L2 left to everything else)
     if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
+    // hub cache: entries per rank block (needed for the BFS kernel's shared memory)
+    {
+        int hc = cfg.hub_cache;
+        if (hc < 0) hc = 0;   // auto = off: measured slower than the L1 on RMAT-24/26 (DESIGN.md "hub cache")
+        hc -= hc % (32 * g->p);
+        g->hc_per_rank = hc / g->p;
+    }
+    const int want = cfg.ctas_per_sm > 0 ? cfg.ctas_per_sm : 1024 / kThreads;
+    const size_t smem_bfs = worker_smem(kApBfs, g->hc_per_rank * g->p), smem_pr = worker_smem(kApPr, 0);
     int occ0 = 0, occ1 = 0, occ2 = 0, occ3 = 0;   // single- and multi-rank specialisations
-    CU((kernel_setup<kApBfs, false>(occ0, worker_smem(kApBfs, kHubMax))));
-    CU((kernel_setup<kApPr, false>(occ1, worker_smem(kApPr, 0))));
-    CU((kernel_setup<kApBfs, true>(occ2, worker_smem(kApBfs, kHubMax))));
-    CU((kernel_setup<kApPr, true>(occ3, worker_smem(kApPr, 0))));
+    CU((kernel_setup<kApBfs, false>(occ0, smem_bfs, want)));
+    CU((kernel_setup<kApPr, false>(occ1, smem_pr, want)));
+    CU((kernel_setup<kApBfs, true>(occ2, smem_bfs, want)));
+    CU((kernel_setup<kApPr, true>(occ3, smem_pr, want)));
     g->occ = std::min(std::min(occ0, occ1), std::min(occ2, occ3));
     if (cfg.ctas_per_sm > 0) g->occ = std::min(g->occ, cfg.ctas_per_sm);
     if (g->occ < 1) return fail(ATOS_ERR_CUDA, "worker kernel cannot be resident (occupancy 0)");
@@ -564,13 +581,6 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (cfg.relabel != 0 && n > 1) {
         atos_status rs = compute_relabel(g, row_ptr, rp_dev);
         if (rs != ATOS_OK) return rs;
-    }
-    // hub cache: entries per rank block
-    {
-        int hc = cfg.hub_cache;
-        if (hc < 0) hc = 0;   // auto = off: measured slower than the L1 on RMAT-24/26 (DESIGN.md "hub cache")
-        hc -= hc % (32 * g->p);
-        g->hc_per_rank = hc / g->p;
     }
 
     unsigned long long *d_bad = nullptr;

@@ -38,26 +38,34 @@ constexpr int kApPr = 1;
 #endif
 constexpr int kU = ATOS_KU;          // edges per lane in flight
 constexpr int kChunk = 32 * kU;      // edges per warp chunk
-constexpr int kWOut = 256;           // per-warp local staging (items)
+#ifndef ATOS_WOUT
+#define ATOS_WOUT 256
+#endif
+constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr int kHubMax = 131072;      // max hub-cache entries per CTA (64 KB of nibbles)
+constexpr int kHubMax = 65536;       // max hub-cache entries per CTA (32 KB of nibbles; 2 CTAs/SM still fit)
 
 template <int APP> struct AppTraits;
 template <> struct AppTraits<kApBfs> { static constexpr int kMsgBytes = 8; };
 template <> struct AppTraits<kApPr> { static constexpr int kMsgBytes = 16; };
 
+// One popped batch, set up for expansion.
+struct BatchBuf {
+    uint32_t v[kThreads];          // local vertex ids
+    uint64_t val[kThreads];        // depth (BFS) or delta bits (PR)
+    int64_t beg[kThreads];         // row begin (offset into col)
+    int64_t off[kThreads + 1];     // exclusive prefix of edge counts
+    uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
+    uint32_t chunk_next;           // next unclaimed edge chunk
+};
+
 struct Smem {
     RankDev R;
-    uint32_t v[kThreads];          // batch: local vertex ids
-    uint64_t val[kThreads];        // batch: depth (BFS) or delta bits (PR)
-    int64_t beg[kThreads];         // batch: row begin (offset into col)
-    int64_t off[kThreads + 1];     // batch: exclusive prefix of edge counts
+    BatchBuf bb[1];
     uint32_t wout[kWarps][kWOut];  // per-warp local push staging
     uint32_t wn[kWarps];
     uint32_t wpre[kWarps + 1];
-    uint32_t chunk_next;           // next unclaimed edge chunk of the batch
-    uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
     uint32_t wst[kWarps][kMaxRanks], wsh[kWarps][kMaxRanks];   // per-warp message staging tail/head
     uint64_t wt0[kWarps][kMaxRanks];                           // time staging became non-empty
     int64_t wsum[kWarps];
@@ -177,10 +185,10 @@ __device__ __forceinline__ int64_t block_exscan(Smem &s, int64_t x, int64_t &exc
 }
 
 // largest j in [lo, hi] with off[j] <= e   (off[lo] <= e holds)
-__device__ __forceinline__ int upper_vertex(const Smem &s, int lo, int hi, int64_t e) {
+__device__ __forceinline__ int upper_vertex(const BatchBuf &bb, int lo, int hi, int64_t e) {
     while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
-        if (s.off[mid] <= e) lo = mid; else hi = mid - 1;
+        if (bb.off[mid] <= e) lo = mid; else hi = mid - 1;
     }
     return lo;
 }
@@ -521,7 +529,7 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
 // batch expansion
 // ---------------------------------------------------------------------------
 template <int APP, bool MULTI>
-__device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
+__device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
     const RankDev &R = s.R;
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // register copies of the hot rank fields (s.R lives in smem)
@@ -535,7 +543,7 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
     for (;;) {
         // dynamic chunk claim: a warp that finishes early takes the next chunk
         uint32_t c = 0;
-        if (lane == 0) c = atomicAdd(&s.chunk_next, 1u);
+        if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
         c = __shfl_sync(kFull, c, 0);
         if (c >= nch) break;
 #ifdef ATOS_PROF
@@ -545,11 +553,11 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
         const int64_t clast = (E < c0 + kChunk ? E : c0 + kChunk) - 1;
         int jlo, jhi;
         if (c + 1 < (uint32_t)kChunkMap) {      // precomputed in process_batch
-            jlo = s.chunk_v[c];
-            jhi = c + 1 < nch ? s.chunk_v[c + 1] : B - 1;
+            jlo = bb.chunk_v[c];
+            jhi = c + 1 < nch ? bb.chunk_v[c + 1] : B - 1;
         } else {
-            jlo = upper_vertex(s, s.off[jprev] <= c0 ? jprev : 0, B - 1, c0);
-            jhi = upper_vertex(s, jlo, B - 1, clast);
+            jlo = upper_vertex(bb, bb.off[jprev] <= c0 ? jprev : 0, B - 1, c0);
+            jhi = upper_vertex(bb, jlo, B - 1, clast);
         }
         jprev = jlo;
         int j = jlo;
@@ -562,12 +570,12 @@ __device__ void expand_warp(Smem &s, const KParams &kp, int cta, int B, int64_t 
             u[k] = -1;
             vv[k] = 0;
             if (e <= clast) {
-                if (j < jhi && s.off[j + 1] <= e) {       // usually one step for skewed graphs
+                if (j < jhi && bb.off[j + 1] <= e) {       // usually one step for skewed graphs
                     ++j;
-                    if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
+                    if (j < jhi && bb.off[j + 1] <= e) j = upper_vertex(bb, j + 1, jhi, e);
                 }
-                u[k] = ld_stream(col + s.beg[j] + (e - s.off[j]), pol);
-                vv[k] = (ValT)s.val[j];
+                u[k] = ld_stream(col + bb.beg[j] + (e - bb.off[j]), pol);
+                vv[k] = (ValT)bb.val[j];
             }
         }
 #ifdef ATOS_PROF
@@ -671,7 +679,7 @@ struct PipeStage {
     uint32_t nd[kPU];
 };
 
-__device__ __forceinline__ void pipe_load(const Smem &s, int B, int64_t E, uint32_t nchm, uint32_t c, PipeStage &st,
+__device__ __forceinline__ void pipe_load(const BatchBuf &bb, int B, int64_t E, uint32_t nchm, uint32_t c, PipeStage &st,
                                           const int32_t *col, uint64_t pol) {
     const int lane = threadIdx.x & 31;
     const int64_t c0 = (int64_t)c * kPChunk;
@@ -679,11 +687,11 @@ __device__ __forceinline__ void pipe_load(const Smem &s, int B, int64_t E, uint3
     const uint32_t m = (uint32_t)(c0 / kChunk);          // map chunk containing c0
     int jlo, jhi;
     if (m + 1 < (uint32_t)kChunkMap) {
-        jlo = s.chunk_v[m];                               // vertex of edge m*kChunk <= vertex of c0
-        jhi = m + 1 < nchm ? s.chunk_v[m + 1] : B - 1;
+        jlo = bb.chunk_v[m];                               // vertex of edge m*kChunk <= vertex of c0
+        jhi = m + 1 < nchm ? bb.chunk_v[m + 1] : B - 1;
     } else {
-        jlo = upper_vertex(s, 0, B - 1, c0);
-        jhi = upper_vertex(s, jlo, B - 1, clast);
+        jlo = upper_vertex(bb, 0, B - 1, c0);
+        jhi = upper_vertex(bb, jlo, B - 1, clast);
     }
     int j = jlo;
 #pragma unroll
@@ -692,12 +700,12 @@ __device__ __forceinline__ void pipe_load(const Smem &s, int B, int64_t E, uint3
         st.u[k] = -1;
         st.nd[k] = 0;
         if (e <= clast) {
-            if (j < jhi && s.off[j + 1] <= e) {
+            if (j < jhi && bb.off[j + 1] <= e) {
                 ++j;
-                if (j < jhi && s.off[j + 1] <= e) j = upper_vertex(s, j + 1, jhi, e);
+                if (j < jhi && bb.off[j + 1] <= e) j = upper_vertex(bb, j + 1, jhi, e);
             }
-            st.u[k] = ld_stream(col + s.beg[j] + (e - s.off[j]), pol);
-            st.nd[k] = (uint32_t)s.val[j] + 1u;
+            st.u[k] = ld_stream(col + bb.beg[j] + (e - bb.off[j]), pol);
+            st.nd[k] = (uint32_t)bb.val[j] + 1u;
         }
     }
 }
@@ -724,24 +732,24 @@ __device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, 
 }
 
 template <int APP, bool MULTI>
-__device__ void expand_warp_pipe(Smem &s, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
+__device__ void expand_warp_pipe(Smem &s, BatchBuf &bb, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
     const int lane = threadIdx.x & 31;
     const int32_t *const col = s.R.col;
     const uint64_t pol = policy_evict_first();
     const uint32_t nchm = (uint32_t)((E + kChunk - 1) / kChunk);
     const uint32_t nch = (uint32_t)((E + kPChunk - 1) / kPChunk);
     uint32_t c = 0;
-    if (lane == 0) c = atomicAdd(&s.chunk_next, 1u);
+    if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
     c = __shfl_sync(kFull, c, 0);
     if (c >= nch) return;
     PipeStage a, b;
-    pipe_load(s, B, E, nchm, c, a, col, pol);
+    pipe_load(bb, B, E, nchm, c, a, col, pol);
     for (;;) {
         uint32_t c2 = 0;
-        if (lane == 0) c2 = atomicAdd(&s.chunk_next, 1u);
+        if (lane == 0) c2 = atomicAdd(&bb.chunk_next, 1u);
         c2 = __shfl_sync(kFull, c2, 0);
         const bool more = c2 < nch;
-        if (more) pipe_load(s, B, E, nchm, c2, b, col, pol);   // next chunk's columns in flight
+        if (more) pipe_load(bb, B, E, nchm, c2, b, col, pol);   // next chunk's columns in flight
         pipe_relax<APP, MULTI>(s, kp, cta, a, wn);
         if (!more) break;
         a = b;
@@ -752,42 +760,43 @@ __device__ void expand_warp_pipe(Smem &s, const KParams &kp, int cta, int B, int
 template <int APP, bool MULTI>
 __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     const RankDev &R = s.R;
+    BatchBuf &bb = s.bb[0];
     const int tid = threadIdx.x;
 #ifdef ATOS_PROF
     if (tid == 0) s.prof[7] -= (unsigned long long)clock64();
 #endif
     int64_t deg = 0;
     if (tid < B) {
-        const uint32_t v = s.v[tid];
+        const uint32_t v = bb.v[tid];
         const int64_t b = ldg_i64_nc(R.row_ptr + v), e = ldg_i64_nc(R.row_ptr + v + 1);
-        s.beg[tid] = b;
+        bb.beg[tid] = b;
         deg = e - b;
         if constexpr (APP == kApBfs) {
             // claim the expansion of v at its current depth; stale duplicates see
             // the pending bit already cleared and are skipped
             const uint32_t old = atom_and_u32(R.depth + R.v_begin + v, ~1u);
             const uint32_t d = dw_depth(old);
-            s.val[tid] = d;
+            bb.val[tid] = d;
             if (!(old & 1u) || d == kDepthInf) deg = 0;
         } else {
             const int64_t sl = pr_slot(v, R.pr_q);
             const double r = __longlong_as_double((long long)atom_exch_u64((uint64_t *)(R.pr_res + sl), 0ull));
             if (r != 0.0) red_add_f64(R.pr_rank + sl, r);
             if (r == 0.0 || deg == 0) deg = 0;        // dangling vertices absorb (R4)
-            else s.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
+            else bb.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
         }
     }
-    if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + s.beg[tid], (uint64_t)deg * 4);
+    if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + bb.beg[tid], (uint64_t)deg * 4);
     int64_t excl;
     const int64_t E = block_exscan(s, deg, excl);
     if (tid < B) {
-        s.off[tid] = excl;
+        bb.off[tid] = excl;
         if (deg > 0) {   // chunk -> first vertex map: chunks starting inside this row
             const int64_t cl = (excl + deg - 1) / kChunk;
-            for (int64_t c = (excl + kChunk - 1) / kChunk; c <= cl && c < kChunkMap; ++c) s.chunk_v[c] = (uint16_t)tid;
+            for (int64_t c = (excl + kChunk - 1) / kChunk; c <= cl && c < kChunkMap; ++c) bb.chunk_v[c] = (uint16_t)tid;
         }
     }
-    if (tid == 0) { s.off[B] = E; s.c_edges += (unsigned long long)E; s.chunk_next = 0; }
+    if (tid == 0) { bb.off[B] = E; s.c_edges += (unsigned long long)E; bb.chunk_next = 0; }
     __syncthreads();
 #ifdef ATOS_PROF
     if (tid == 0) s.prof[7] += (unsigned long long)clock64();   // minus entry below: setup+scan
@@ -797,8 +806,8 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         uint32_t wn = s.wn[w];
         // pipelined expansion pays off on low-degree (latency-bound, road-like) batches
         if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
-            expand_warp_pipe<APP, MULTI>(s, kp, cta, B, E, wn);
-        else expand_warp<APP, MULTI>(s, kp, cta, B, E, wn);
+            expand_warp_pipe<APP, MULTI>(s, bb, kp, cta, B, E, wn);
+        else expand_warp<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
@@ -810,6 +819,7 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
 template <int APP, bool MULTI>
 __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
     const int tid = threadIdx.x, w = tid >> 5;
+    BatchBuf &bb = s.bb[0];
     __syncthreads();
     if constexpr (MULTI) {
         uint32_t wn = s.wn[w];
@@ -846,7 +856,7 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
         int k = 0;
         while (k + 1 < kWarps && s.wpre[k + 1] <= i) ++k;
         const uint32_t item = s.wout[k][i - s.wpre[k]];
-        if (i < keep_n) s.v[i] = item;
+        if (i < keep_n) bb.v[i] = item;
         else ring_store(s.R, base + (i - keep_n), item, s.ring_base);
     }
     __syncthreads();
@@ -879,6 +889,7 @@ __device__ void report_staged(Smem &s) {
 __device__ int pop_batch(Smem &s, const KParams &kp) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x;
+    BatchBuf &bb = s.bb[0];
     if (tid == 0) {
         if (s.res_lo == s.res_hi) {
             const uint64_t t = ld_relaxed_gpu(&R.ctrl->tail.v);
@@ -908,7 +919,7 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
     if (tid < B) {
         // no acquire fence: the vertex state is only accessed through L2 atomics
         // whose address depends on this slot value (see warp_flush_local)
-        s.v[tid] = lo32(slot);
+        bb.v[tid] = lo32(slot);
         st_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)], pack(lo32(idx + R.ring_cap), 0u));
     }
     __syncthreads();

@@ -210,7 +210,7 @@ def test_hub_cache_active_on_skewed_graph():
     g = inputs.rmat(16, 16, 1, symmetric=True)
     rp, col = g.numpy()
     src = inputs.bfs_sources(g, 1)[0]
-    with atos.Graph(rp, col, relabel=1, hub_cache=131072) as G:
+    with atos.Graph(rp, col, relabel=1, hub_cache=65536) as G:
         d, st = G.bfs(src, stats=True)
     assert np.array_equal(d, oracle.bfs(rp, col, src))
     assert st["hub_hits"] > 0.2 * st["edges"], st
