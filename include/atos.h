@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define ATOS_ABI_VERSION 2
+#define ATOS_ABI_VERSION 3
 #define ATOS_MAX_RANKS 8          /* one NVSwitch box: 8 GPUs */
 #define ATOS_IPC_HANDLE_BYTES 64  /* == sizeof(cudaIpcMemHandle_t) */
 
@@ -56,8 +56,11 @@ typedef struct {
     int32_t fetch_size;       /* max vertices popped per worker batch (the
                                  paper's FETCH_SIZE); <= worker_threads */
     int32_t keep_items;       /* max discovered vertices a worker keeps as its
-                                 own next batch when the ring is nearly empty
-                                 (work-keeping; 0 = always enqueue); <= 512    */
+                                 own next batch instead of enqueueing them
+                                 (work-keeping; 0 = always enqueue; <= 512);
+                                 -1 = auto: 128 with keep_mode 1 on graphs that
+                                 are not skewed (high-diameter, road-like), 0 on
+                                 skewed ones        */
     int32_t l2_persist;       /* 1: give the random-access state (BFS words /
                                  PR residuals) an L2 persisting access-policy
                                  window during the worker kernel; sets the
@@ -99,6 +102,35 @@ typedef struct {
                                  x n_ranks, <= 65536; 0 = off; -1 = auto
                                  (currently off: the L1 already serves hub
                                  probes; kept as a measured option)           */
+    int32_t split_edges;      /* BFS: a popped row longer than 2 x split_edges
+                                 is cut into split_edges-edge pieces that any
+                                 worker can pop (the popping worker keeps the
+                                 first); only for the first 65536 ids of a rank
+                                 block (the hubs after relabeling).  Power of
+                                 two in [256, 1<<20]; 0 = off; -1 = auto       */
+    int32_t keep_mode;        /* when a worker keeps (keep_items > 0): 0 = only
+                                 while the rank's outstanding work is <=
+                                 keep_items (low-parallelism phases), 1 =
+                                 whenever its batch discovered <= keep_items
+                                 (latency chains; may add redundant work).
+                                 Ignored when keep_items == -1 (auto)         */
+    int32_t discrete;         /* 0 = one persistent worker kernel per solve
+                                 (the paper's default); 1 = discrete
+                                 kernels: each launch
+                                 processes the queue snapshot [head, tail) and
+                                 exits; a CUDA-graph while-node relaunches it
+                                 until the queue is empty, with no host round
+                                 trip.  Single rank only (n_ranks == 1 and
+                                 virtual_ranks == 1)                           */
+    int32_t pr_combine;       /* PageRank, n_ranks > 1 (not in the
+                                 paper): 1 = sender-side residual combining --
+                                 deltas for a remote vertex accumulate in this
+                                 rank's ghost residual, which is sent as ONE
+                                 message when it crosses eps / n_ranks; the
+                                 returned residual then includes the unsent
+                                 ghost mass (< eps in total per vertex beyond
+                                 the owner's own < eps).  0 = send every delta
+                                 (the paper's push, with aggregation)          */
 } atos_config;
 
 /* Per-solve statistics (device counters, summed over the ranks this handle
@@ -118,6 +150,7 @@ typedef struct {
                                  cache without an L2 probe                    */
     uint64_t busy_ns;         /* sum over workers of time spent on work (ns)   */
     uint64_t batches;         /* work units (pop batches + packets + chunks)   */
+    uint64_t iterations;      /* discrete mode: worker launches in the solve   */
     int32_t n_ranks;          /* ranks covered by these counters               */
     int32_t grid_ctas;        /* persistent CTAs per rank                      */
 } atos_stats;

@@ -51,6 +51,10 @@ class Config(ctypes.Structure):
         ("stream", ctypes.c_void_p),
         ("relabel", ctypes.c_int32),
         ("hub_cache", ctypes.c_int32),
+        ("split_edges", ctypes.c_int32),
+        ("keep_mode", ctypes.c_int32),
+        ("discrete", ctypes.c_int32),
+        ("pr_combine", ctypes.c_int32),
     ]
 
 
@@ -68,6 +72,7 @@ class Stats(ctypes.Structure):
         ("hub_hits", ctypes.c_uint64),
         ("busy_ns", ctypes.c_uint64),
         ("batches", ctypes.c_uint64),
+        ("iterations", ctypes.c_uint64),
         ("n_ranks", ctypes.c_int32),
         ("grid_ctas", ctypes.c_int32),
     ]

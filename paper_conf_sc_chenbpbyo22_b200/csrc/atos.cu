@@ -45,6 +45,22 @@ static atos_status fail(atos_status st, const char *fmt, ...) {
         }                                                                                         \
     } while (0)
 
+// Opt-in phase trace of graph_load (ATOS_LOAD_TRACE=1): syncs the stream at each
+// mark and prints the host wall time of the phase to stderr.  Diagnostic only.
+#include <chrono>
+#include <cstdlib>
+struct LoadTrace {
+    bool on = std::getenv("ATOS_LOAD_TRACE") != nullptr;
+    std::chrono::steady_clock::time_point t = std::chrono::steady_clock::now();
+    void mark(cudaStream_t st, const char *what) {
+        if (!on) return;
+        cudaStreamSynchronize(st);
+        const auto now = std::chrono::steady_clock::now();
+        fprintf(stderr, "[atos load] %-24s %8.2f ms\n", what, std::chrono::duration<double, std::milli>(now - t).count());
+        t = now;
+    }
+};
+
 extern "C" const char *atos_last_error(void) { return g_err; }
 extern "C" int32_t atos_version(void) { return ATOS_ABI_VERSION; }
 
@@ -57,7 +73,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->worker_threads = kThreads;
     cfg->ctas_per_sm = 0;
     cfg->fetch_size = kThreads;
-    cfg->keep_items = 0;
+    cfg->keep_items = -1;
     cfg->l2_persist = 1;
     cfg->prefetch = 0;    // measured slower on RMAT-24 with both worker modes
     cfg->relax_red = 1;
@@ -76,6 +92,8 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->stream = nullptr;
     cfg->relabel = 2;
     cfg->hub_cache = -1;
+    cfg->split_edges = -1;
+    cfg->pr_combine = 0;
     return ATOS_OK;
 }
 
@@ -101,21 +119,25 @@ extern "C" atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *
 static bool valid_cfg(const atos_config &c) {
     auto pow2 = [](int64_t x) { return x > 0 && (x & (x - 1)) == 0; };
     return c.worker_threads == kThreads && c.fetch_size >= 1 && c.fetch_size <= kThreads &&
-           c.keep_items >= 0 && c.keep_items <= kThreads &&
+           c.keep_items >= -1 && c.keep_items <= kThreads && (c.keep_mode == 0 || c.keep_mode == 1) &&
            c.ring_cap_factor >= 1.0 && c.agg_batch_msgs >= 1 && c.agg_batch_msgs <= 4096 &&
            c.agg_max_age_ns >= 0 && pow2(c.channel_packets) && c.channel_packets <= (1 << 20) &&
            c.watchdog_ms >= 0 && c.n_ranks >= 1 && c.n_ranks <= ATOS_MAX_RANKS && c.rank >= 0 &&
            c.rank < c.n_ranks && c.virtual_ranks >= 1 && c.virtual_ranks <= ATOS_MAX_RANKS &&
            !(c.virtual_ranks > 1 && c.n_ranks > 1) && c.ctas_per_sm >= 0 && c.device >= 0 &&
            c.relabel >= 0 && c.relabel <= 2 && c.hub_cache >= -1 && c.hub_cache <= kHubMax &&
-           (c.hub_cache <= 0 || c.hub_cache % (32 * std::max(c.n_ranks, c.virtual_ranks)) == 0);
+           (c.hub_cache <= 0 || c.hub_cache % (32 * std::max(c.n_ranks, c.virtual_ranks)) == 0) &&
+           (c.split_edges == 0 || c.split_edges == -1 ||
+            (c.split_edges >= 256 && c.split_edges <= (1 << 20) && pow2(c.split_edges))) &&
+           (c.pr_combine == 0 || c.pr_combine == 1) &&
+           (c.discrete == 0 || (c.discrete == 1 && c.n_ranks == 1 && c.virtual_ranks == 1));
 }
 
 // ---------------------------------------------------------------------------
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, filt, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, total;
+    size_t ctrl, depth, filt, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, ghost, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -131,6 +153,7 @@ struct Shape {
     int p;
     int cp, pkt, stage_cap, ctas_per_rank, fetch;
     double ring_factor;
+    int combine;       // PR ghost residuals allocated (n_ranks > 1 && pr_combine)
 };
 
 static Layout make_layout(const Shape &S, const int64_t *part, int r) {
@@ -152,6 +175,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.free_m = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
     L.staging = o; o = al(o + (multi ? (size_t)S.ctas_per_rank * kWarps * kMaxRanks * S.stage_cap * 16 : 0));
     L.parent = o;  o = al(o + (size_t)S.n * 8);
+    L.ghost = o;   o = al(o + (multi && S.combine ? (size_t)S.n * 8 : 0));
     L.total = o;
     return L;
 }
@@ -168,7 +192,7 @@ struct LocalRank {
     int64_t *row_ptr = nullptr;
     int32_t *col = nullptr;
     int64_t m_r = 0;
-    uint64_t snap[9] = {0};   // stat counters after the previous solve
+    uint64_t snap[10] = {0};  // stat counters after the previous solve
 };
 
 struct atos_graph {
@@ -193,6 +217,7 @@ struct atos_graph {
     int32_t *d_perm = nullptr;     // degree relabeling: old -> new (NULL = identity)
     int32_t *d_inv = nullptr;      //                    new -> old
     int hc_per_rank = 0;           // BFS hub-cache entries per rank block
+    bool skewed = true;            // max degree >= 32 x mean degree (set when an auto option needs it)
     int64_t **d_accs = nullptr;
     uint64_t epoch = 0;
     cudaEvent_t ev_begin = nullptr, ev_w0 = nullptr, ev_w1 = nullptr, ev_end = nullptr;
@@ -200,6 +225,11 @@ struct atos_graph {
     int app = kApBfs;          // application of the pending / last solve
     atos_stats last{};
     bool last_valid = false;
+    // discrete-kernel mode: per-app instantiated graph
+    // [step -> while(queue non-empty){ worker -> step }], parameters in d_kp
+    KParams *d_kp = nullptr;
+    cudaGraph_t dgraph[2] = {nullptr, nullptr};
+    cudaGraphExec_t dexec[2] = {nullptr, nullptr};
 };
 
 // dynamic shared memory of the worker: Smem, plus the BFS hub cache (one nibble per entry)
@@ -210,17 +240,20 @@ static size_t worker_smem(int app, int hc_entries) {
 // Dynamic smem limit, then the smallest shared-memory carve-out that still holds
 // `want` CTAs per SM: the rest of the 256 KB unified L1/smem stays L1, which caches
 // the hot (relabeled) part of the BFS depth words -- measured to matter.
-template <int APP, bool MULTI>
-static cudaError_t kernel_setup(int &occ, size_t smem, int want) {
-    cudaError_t e = cudaFuncSetAttribute(worker_kernel<APP, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem);
+template <typename F>
+static cudaError_t kernel_setup_fn(F *fn, int &occ, size_t smem, int want) {
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    const double need_kb = (double)want * ((double)(smem + 1024 + 1024) / 1024.0);   // + static + reserved
+    const double need_kb = (double)want * ((double)(smem + sizeof(KParams) + 1024 + 1024) / 1024.0);   // + static + reserved
     int pct = (int)(need_kb / 228.0 * 100.0) + 1;
     pct = pct > 100 ? 100 : pct;
-    e = cudaFuncSetAttribute(worker_kernel<APP, MULTI>, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
     if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, worker_kernel<APP, MULTI>, kThreads, smem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kThreads, smem);
+}
+template <int APP, bool MULTI>
+static cudaError_t kernel_setup(int &occ, size_t smem, int want) {
+    return kernel_setup_fn(worker_kernel<APP, MULTI>, occ, smem, want);
 }
 
 static RankDev build_view(const atos_graph *g, int lr) {
@@ -242,6 +275,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     d.pr_rank = (double *)(b + L.rank);
     d.pr_res = (double *)(b + L.res);
     d.pr_q = pr_q_of(L.n_r);
+    d.pr_ghost = (g->p > 1 && g->S.combine) ? (double *)(b + L.ghost) : nullptr;
     d.ring = (uint64_t *)(b + L.ring);
     d.ring_cap = L.ring_cap;
     d.ctrl = (Ctrl *)(b + L.ctrl);
@@ -260,6 +294,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
         d.peer_depth[s] = (uint32_t *)(bs + Ls.depth);
         d.peer_rank[s] = (double *)(bs + Ls.rank);
         d.peer_res[s] = (double *)(bs + Ls.res);
+        d.peer_ghost[s] = (g->p > 1 && g->S.combine) ? (double *)(bs + Ls.ghost) : nullptr;
         if (g->p > 1) {
             d.in_hdr[s] = (uint64_t *)(b + L.in_hdr + (size_t)s * cp * 8);
             d.in_payload[s] = b + L.in_pay + (size_t)s * cp * pkt * 16;
@@ -375,6 +410,11 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     cudaFree(g->d_perm);
     cudaFree(g->d_inv);
     cudaFree(g->d_accs);
+    for (int a = 0; a < 2; ++a) {
+        if (g->dexec[a]) cudaGraphExecDestroy(g->dexec[a]);
+        if (g->dgraph[a]) cudaGraphDestroy(g->dgraph[a]);
+    }
+    cudaFree(g->d_kp);
     if (g->ev_begin) cudaEventDestroy(g->ev_begin);
     if (g->ev_w0) cudaEventDestroy(g->ev_w0);
     if (g->ev_w1) cudaEventDestroy(g->ev_w1);
@@ -400,7 +440,7 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
     else atos_partition_balanced(n, n_ranks, pt.data());
     Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs),
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
-            cfg.fetch_size, cfg.ring_cap_factor};
+            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine};
     *bytes_out = make_layout(S, pt.data(), rank).total;
     return ATOS_OK;
 }
@@ -437,10 +477,10 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     unsigned long long mx = 0;
     CU(cudaMemcpyAsync(&mx, d_max, 8, cudaMemcpyDeviceToHost, st));
     CU(cudaStreamSynchronize(st));
-    if (g->cfg.relabel == 2) {
-        const double mean = (double)g->nnz / (double)n;
-        if (!((double)mx >= 32.0 * std::max(1.0, mean))) return ATOS_OK;   // not skewed: keep the given order
-    }
+    const double mean = (double)g->nnz / (double)n;
+    g->skewed = (double)mx >= 32.0 * std::max(1.0, mean);
+    if (g->cfg.relabel == 0) return ATOS_OK;                           // degree statistics only
+    if (g->cfg.relabel == 2 && !g->skewed) return ATOS_OK;              // not skewed: keep the given order
     CU(cudaMalloc(&g->d_inv, (size_t)n * 4));
     CU(cudaMalloc(&g->d_perm, (size_t)n * 4));
     int64_t maxlen = 0;
@@ -558,6 +598,12 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     CU((kernel_setup<kApBfs, true>(occ2, smem_bfs, want)));
     CU((kernel_setup<kApPr, true>(occ3, smem_pr, want)));
     g->occ = std::min(std::min(occ0, occ1), std::min(occ2, occ3));
+    if (cfg.discrete) {
+        int occ4 = 0, occ5 = 0;
+        CU(kernel_setup_fn(worker_discrete_kernel<kApBfs>, occ4, smem_bfs, want));
+        CU(kernel_setup_fn(worker_discrete_kernel<kApPr>, occ5, smem_pr, want));
+        g->occ = std::min(g->occ, std::min(occ4, occ5));
+    }
     if (cfg.ctas_per_sm > 0) g->occ = std::min(g->occ, cfg.ctas_per_sm);
     if (g->occ < 1) return fail(ATOS_ERR_CUDA, "worker kernel cannot be resident (occupancy 0)");
     const int ctas_total = g->occ * g->sms;
@@ -565,7 +611,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
     g->grid = cpr * g->n_local;
     g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs), cpr,
-                 cfg.fetch_size, cfg.ring_cap_factor};
+                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine};
 
     if (cfg.stream) {
         g->stream = (cudaStream_t)cfg.stream;
@@ -578,8 +624,11 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     CU(cudaEventCreate(&g->ev_w1));
     CU(cudaEventCreate(&g->ev_end));
 
-    if (cfg.relabel != 0 && n > 1) {
+    LoadTrace tr;
+    tr.mark(g->stream, "setup");
+    if ((cfg.relabel != 0 || cfg.keep_items < 0) && n > 1) {
         atos_status rs = compute_relabel(g, row_ptr, rp_dev);
+        tr.mark(g->stream, "compute_relabel");
         if (rs != ATOS_OK) return rs;
     }
 
@@ -595,13 +644,16 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         me.m_r = rb[r + 1] - rb[r];
         CU(cudaMalloc(&me.arena, me.L.total));
         CU(cudaMemsetAsync(me.arena, 0, me.L.total, g->stream));
+        tr.mark(g->stream, "arena");
         CU(cudaMalloc(&me.row_ptr, (size_t)(nr + 1) * 8));
         CU(cudaMalloc(&me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
         CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
         if (me.m_r > 0)
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
+        tr.mark(g->stream, "copy csr");
         rebase_rows_kernel<<<256, 256, 0, g->stream>>>(me.row_ptr, nr + 1, rb[r]);
         check_rows_kernel<<<1024, 256, 0, g->stream>>>(me.row_ptr, nr, me.m_r, me.col, n, d_bad);
+        tr.mark(g->stream, "check rows");
         if (g->d_perm) {   // rows must be valid before they are permuted
             unsigned long long bad0 = 0;
             CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
@@ -609,6 +661,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
             if (bad0) { cudaFree(d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: invalid row_ptr or column index"); }
             atos_status rs = relabel_rows(g, me);
             if (rs != ATOS_OK) { cudaFree(d_bad); return rs; }
+            tr.mark(g->stream, "relabel rows");
         }
         const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
         init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
@@ -628,6 +681,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     g->connected = !g->multiproc;
     atos_status st = upload_views(g);
     if (st != ATOS_OK) return st;
+    tr.mark(g->stream, "finish");
     guard.g = nullptr;
     *out = g;
     return ATOS_OK;
@@ -678,7 +732,8 @@ static KParams make_params(atos_graph *g) {
     kp.cp = g->S.cp;
     kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
-    kp.keep = g->cfg.keep_items;
+    kp.keep = g->cfg.keep_items >= 0 ? g->cfg.keep_items : (g->skewed ? 0 : kKeepAuto);
+    kp.keep_always = g->cfg.keep_items >= 0 ? g->cfg.keep_mode : 1;
     kp.prefetch = g->cfg.prefetch;
     kp.relax_red = g->cfg.relax_red;
     kp.pipe = g->cfg.pipeline;
@@ -687,14 +742,104 @@ static KParams make_params(atos_graph *g) {
     kp.filter = g->cfg.probe_filter == 1 ||
                 (g->cfg.probe_filter == 2 && (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20));
     kp.hc_per_rank = g->hc_per_rank;
+    kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
+    kp.combine = g->p > 1 && g->S.combine;
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;
     return kp;
 }
 
+// L2 persisting window for the random-access state of the worker (BFS words or
+// filter / PR residuals); sets the device's persisting carve-out to match.
+// Returns false when no window applies.
+template <int APP>
+static bool l2_window(atos_graph *g, const KParams &kp, cudaAccessPolicyWindow &w) {
+    if (!(g->cfg.l2_persist && g->n_local == 1 && g->persist_max > 0 && g->window_max > 0)) return false;
+    // keep the random-access state resident in L2 while the CSR column stream
+    // passes through
+    const LocalRank &me = g->loc[0];
+    void *base = APP == kApBfs ? (void *)(me.arena + (kp.filter ? me.L.filt : me.L.depth))
+                               : (void *)(me.arena + me.L.res);
+    size_t bytes = APP == kApBfs ? (size_t)g->n * (kp.filter ? 1 : 4) : (size_t)me.L.n_r * 8;
+    bytes = std::min(bytes, g->window_max);
+    const size_t carve = std::min(bytes, g->persist_max);   // carve-out == window, no more
+    if (carve != g->persist_set) {
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve) != cudaSuccess) {
+            cudaGetLastError();
+            g->persist_max = 0;                              // not permitted: no window from now on
+            return false;
+        }
+        g->persist_set = carve;
+    }
+    w.base_ptr = base;
+    w.num_bytes = bytes;
+    w.hitRatio = (float)std::min(1.0, (double)carve / (double)bytes);
+    w.hitProp = cudaAccessPropertyPersisting;
+    w.missProp = cudaAccessPropertyStreaming;
+    return true;
+}
+
+// Build (once per handle and app) the discrete-mode graph:
+//   step -> while (cond) { worker_discrete -> step }
+// step snapshots tail into ctrl->limit and sets cond = (queue non-empty).
+template <int APP>
+static atos_status build_discrete_graph(atos_graph *g, const KParams &kp) {
+    if (g->dexec[APP]) return ATOS_OK;
+    if (!g->d_kp) CU(cudaMalloc(&g->d_kp, sizeof(KParams)));
+    cudaGraph_t gr = nullptr;
+    CU(cudaGraphCreate(&gr, 0));
+    g->dgraph[APP] = gr;
+    cudaGraphConditionalHandle h;
+    CU(cudaGraphConditionalHandleCreate(&h, gr, 1, cudaGraphCondAssignDefault));
+    KParams *dkp = g->d_kp;
+    int first = 0, after = 1;
+    void *step_args[] = {&dkp, &h, &first};
+    void *step_args_after[] = {&dkp, &h, &after};
+    cudaKernelNodeParams sk{};
+    sk.func = (void *)discrete_step_kernel;
+    sk.gridDim = dim3(1);
+    sk.blockDim = dim3(32);
+    sk.kernelParams = step_args;
+    cudaGraphNode_t pre = nullptr, cond = nullptr, wnode = nullptr, post = nullptr;
+    CU(cudaGraphAddKernelNode(&pre, gr, nullptr, 0, &sk));
+    cudaGraphNodeParams cp{};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = h;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    CU(cudaGraphAddNode(&cond, gr, &pre, 1, &cp));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+    void *w_args[] = {&dkp};
+    cudaKernelNodeParams wk{};
+    wk.func = (void *)worker_discrete_kernel<APP>;
+    wk.gridDim = dim3(g->grid);
+    wk.blockDim = dim3(kThreads);
+    wk.sharedMemBytes = (unsigned)worker_smem(APP, kp.hc_per_rank * g->p);
+    wk.kernelParams = w_args;
+    CU(cudaGraphAddKernelNode(&wnode, body, nullptr, 0, &wk));
+    cudaAccessPolicyWindow win{};
+    if (l2_window<APP>(g, kp, win)) {
+        cudaKernelNodeAttrValue av{};
+        av.accessPolicyWindow = win;
+        CU(cudaGraphKernelNodeSetAttribute(wnode, cudaKernelNodeAttributeAccessPolicyWindow, &av));
+    }
+    sk.kernelParams = step_args_after;
+    CU(cudaGraphAddKernelNode(&post, body, &wnode, 1, &sk));
+    CU(cudaGraphInstantiate(&g->dexec[APP], gr, 0));
+    return ATOS_OK;
+}
+
 template <int APP>
 static atos_status launch_worker(atos_graph *g, KParams &kp) {
+    if (g->cfg.discrete) {
+        kp.discrete = 1;
+        atos_status s = build_discrete_graph<APP>(g, kp);
+        if (s != ATOS_OK) return s;
+        CU(cudaMemcpyAsync(g->d_kp, &kp, sizeof(KParams), cudaMemcpyHostToDevice, g->stream));
+        CU(cudaGraphLaunch(g->dexec[APP], g->stream));
+        return ATOS_OK;
+    }
     cudaLaunchConfig_t lc{};
     lc.gridDim = dim3(g->grid);
     lc.blockDim = dim3(kThreads);
@@ -705,29 +850,10 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
     at[na].id = cudaLaunchAttributeCooperative;          // co-residency of the persistent grid
     at[na].val.cooperative = 1;
     ++na;
-    if (g->cfg.l2_persist && g->n_local == 1 && g->persist_max > 0 && g->window_max > 0) {
-        // keep the random-access state (BFS words / PR residuals) resident in L2
-        // while the CSR column stream passes through
-        const LocalRank &me = g->loc[0];
-        void *base = APP == kApBfs ? (void *)(me.arena + (kp.filter ? me.L.filt : me.L.depth))
-                                   : (void *)(me.arena + me.L.res);
-        size_t bytes = APP == kApBfs ? (size_t)g->n * (kp.filter ? 1 : 4) : (size_t)me.L.n_r * 8;
-        bytes = std::min(bytes, g->window_max);
-        const size_t carve = std::min(bytes, g->persist_max);   // carve-out == window, no more
-        if (carve != g->persist_set) {
-            if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve) != cudaSuccess) {
-                cudaGetLastError();
-                g->persist_max = 0;                              // not permitted: no window from now on
-            } else {
-                g->persist_set = carve;
-            }
-        }
+    cudaAccessPolicyWindow win{};
+    if (l2_window<APP>(g, kp, win)) {
         at[na].id = cudaLaunchAttributeAccessPolicyWindow;
-        at[na].val.accessPolicyWindow.base_ptr = base;
-        at[na].val.accessPolicyWindow.num_bytes = bytes;
-        at[na].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)carve / (double)bytes);
-        at[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        at[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        at[na].val.accessPolicyWindow = win;
         ++na;
     }
     lc.attrs = at;
@@ -743,7 +869,7 @@ static atos_status read_ctrl(atos_graph *g, int lr, Ctrl &c) {
 }
 
 // Wait for the enqueued solve, check device error flags, fill g->last.
-static constexpr int kSnap = 9;
+static constexpr int kSnap = 10;
 
 static atos_status finish_solve(atos_graph *g) {
     const int app = g->app;
@@ -766,7 +892,7 @@ static atos_status finish_solve(atos_graph *g) {
         if (c.error.v && !err) err = c.error.v;
         const uint64_t now[kSnap] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
                                      c.st_packets.v, c.st_idle.v, c.st_hub_hits.v, c.st_busy_ns.v,
-                                     c.st_batches.v};
+                                     c.st_batches.v, c.st_waves.v};
         uint64_t *sn = g->loc[lr].snap;
         st.pops += now[0] - sn[0];
         st.edges += now[1] - sn[1];
@@ -777,6 +903,7 @@ static atos_status finish_solve(atos_graph *g) {
         st.hub_hits += now[6] - sn[6];
         st.busy_ns += now[7] - sn[7];
         st.batches += now[8] - sn[8];
+        if (g->cfg.discrete) st.iterations += now[9] - sn[9];
         std::memcpy(sn, now, sizeof(now));
     }
     st.bytes_sent = st.msgs_sent * (uint64_t)(app == kApBfs ? AppTraits<kApBfs>::kMsgBytes
@@ -893,6 +1020,7 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     if (s != ATOS_OK) return s;
     kp.alpha = alpha;
     kp.eps = eps;
+    kp.eps_g = eps / (double)g->p;
     const int gblocks = g->sms * 4;
     init_pr_kernel<<<gblocks, 512, 0, g->stream>>>(kp);
     bump_tail_kernel<<<1, 1, 0, g->stream>>>(kp);

@@ -74,6 +74,10 @@ __global__ void init_pr_kernel(KParams kp) {
             const uint64_t idx = base + (uint64_t)i;
             R.ring[idx & (R.ring_cap - 1)] = pack(lo32(idx + 1), (uint32_t)i);
         }
+        if (R.pr_ghost) {   // combining: no unsent residual for any remote vertex
+            for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < R.n; i += (int64_t)gridDim.x * blockDim.x)
+                R.pr_ghost[i] = 0.0;
+        }
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
 }
@@ -127,9 +131,18 @@ __global__ void gather_pr_kernel(KParams kp, double *rank_out, double *res_out) 
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         int o = 0;
         for (int k = 1; k < R.n_ranks; ++k) o += R.part[k] <= v ? 1 : 0;
-        const int64_t i = pr_slot((R.perm ? R.perm[v] : v) - R.part[o], pr_q_of(R.part[o + 1] - R.part[o]));
+        const int64_t nv = R.perm ? R.perm[v] : v;
+        const int64_t i = pr_slot(nv - R.part[o], pr_q_of(R.part[o + 1] - R.part[o]));
         if (rank_out) rank_out[v] = __ldcg(R.peer_rank[o] + i);
-        if (res_out) res_out[v] = __ldcg(R.peer_res[o] + i);
+        if (res_out) {
+            double r = __ldcg(R.peer_res[o] + i);
+            if (R.pr_ghost) {   // combining: unsent ghost mass of every other rank belongs to v's residual
+                const int64_t gi = pr_slot(nv, pr_q_of(n));
+                for (int k = 0; k < R.n_ranks; ++k)
+                    if (k != o) r += __ldcg(R.peer_ghost[k] + gi);
+            }
+            res_out[v] = r;
+        }
     }
 }
 

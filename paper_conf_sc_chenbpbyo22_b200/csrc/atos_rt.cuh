@@ -185,6 +185,7 @@ struct Ctrl {
     Line out_reserve[kMaxRanks]; // packets reserved on channel (this -> d)
     Line in_cursor[kMaxRanks];   // next packet to consume on channel (s -> this)
     Line ring_base;              // tail at the start of the current solve
+    Line limit;                  // discrete mode: queue snapshot this launch may pop up to
     Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_hits, st_waves;
     Line st_busy_ns, st_batches;
 };
@@ -202,6 +203,7 @@ struct RankDev {
     uint8_t *filt;               // BFS: [n] probe filter, an upper bound of depth saturated at 255
     double *pr_rank;             // PR: [n_r], stored at pr_slot(local id)
     double *pr_res;              // PR: [n_r], stored at pr_slot(local id)
+    double *pr_ghost;            // PR combining: [n] unsent residual for remote vertices, at pr_slot(global id, pr_q_of(n)); NULL = off
     int64_t pr_q;                // PR slot spreading: n_r / 8 (0 = identity), see pr_slot
     // local ring (own memory)
     uint64_t *ring;
@@ -225,6 +227,7 @@ struct RankDev {
     uint32_t *peer_depth[kMaxRanks];
     double *peer_rank[kMaxRanks];
     double *peer_res[kMaxRanks];
+    double *peer_ghost[kMaxRanks];
 };
 
 struct KParams {
@@ -237,15 +240,20 @@ struct KParams {
     int32_t stage_cap;       // staging capacity per (cta, warp, dst), messages (pow2)
     int32_t agg_on;
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
+    int32_t keep_always;     // 1: keep whenever <= keep discovered; 0: only when the rank's T - F <= keep
     int32_t prefetch;        // TMA bulk-prefetch each popped adjacency list into L2
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)
     int32_t filter;          // BFS: probe the u8 filter instead of the depth words
     int32_t hc_per_rank;     // BFS hub cache: entries per rank block (0 = off)
+    int32_t split;           // BFS row pieces: edges per piece (0 = off), see kPieceBit
+    int32_t combine;         // PR sender-side residual combining (multi-rank)
+    int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;
     double alpha, eps;       // PageRank
+    double eps_g;            // PR combining: a ghost residual is sent when it crosses eps_g = eps / n_ranks
 };
 
 // ---------------------------------------------------------------------------

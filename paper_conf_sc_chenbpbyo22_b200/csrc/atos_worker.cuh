@@ -21,9 +21,9 @@
 //      per-warp message staging that warps publish to the owner's channel as
 //      packets with one-sided stores over NVLink (aggregation by size / age,
 //      PAPER.md:995-1065).  At batch end the CTA enqueues its discoveries with
-//      one leader atomic, or keeps up to `keep` of them as its next batch when
-//      the ring is nearly empty (work-keeping chain: latency-bound graphs never
-//      round-trip through the queue).
+//      one leader atomic, or keeps up to `keep` of them as its next batch
+//      (work-keeping chain: on latency-bound, high-diameter graphs a worker
+//      follows its own discoveries without a queue round trip per level).
 //   3. idle: flush aged staging, termination detection (single rank: F == T;
 //      multi-rank: coordinator double wave), watchdog.
 #pragma once
@@ -45,6 +45,24 @@ constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr int kHubMax = 65536;       // max hub-cache entries per CTA (32 KB of nibbles; 2 CTAs/SM still fit)
+
+// BFS row pieces.  A popped row longer than
+// 2 x kp.split edges is cut: the popping worker expands the first kp.split edges
+// and publishes the rest as ring items {1 | piece:15 | v:16} that any worker can
+// pop, so a hub's adjacency list is scanned by many CTAs at once instead of
+// serialising one of them.  Only ids < 2^16 of a rank block can be split -- after
+// degree relabeling these are the block's highest-degree vertices.
+constexpr uint32_t kPieceBit = 0x80000000u;
+constexpr int64_t kPieceVMax = 1 << 16;
+constexpr int64_t kPieceMax = 1 << 15;
+constexpr int kKeepAuto = 128;       // work keeping on non-skewed graphs: measured best of 16..512 on the grid
+constexpr int kSplitAuto = 1024;        // measured best of 512..8192 on RMAT-24/26
+
+// PageRank sender-side residual combining (atos_config.pr_combine).
+// A delta for a remote vertex u is added to this rank's ghost residual g[u]; the
+// add that crosses eps_g (the local crossing rule R5 applied to g) exchanges g[u]
+// with 0 and sends the accumulated value as one message.  Deltas below eps_g are
+// thereby combined; quiescence leaves every g[u] < eps_g.
 
 template <int APP> struct AppTraits;
 template <> struct AppTraits<kApBfs> { static constexpr int kMsgBytes = 8; };
@@ -70,6 +88,7 @@ struct Smem {
     uint64_t wt0[kWarps][kMaxRanks];                           // time staging became non-empty
     int64_t wsum[kWarps];
     uint64_t res_lo, res_hi;       // outstanding ring reservation
+    uint64_t limit;                // discrete mode: this launch pops indices < limit
     uint64_t ring_base;            // ring tail at the start of this solve
     uint64_t b64[4];
     int32_t b32[4];
@@ -78,6 +97,10 @@ struct Smem {
     uint64_t staged_reported;
     uint64_t wave[kMaxRanks][5];   // coordinator double wave
     int32_t wave_valid;
+    // CTA-cooperative inbound claim (cta_inbound)
+    int32_t in_got, in_src, in_r;
+    uint64_t in_cc;
+    uint32_t in_off[33];
     unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
 #ifdef ATOS_PROF
     unsigned long long prof[10];
@@ -311,11 +334,13 @@ __device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int
         if constexpr (APP == kApBfs) ((uint64_t *)dpay)[i] = ((const uint64_t *)src)[q];
         else ((uint4 *)dpay)[i] = ((const uint4 *)src)[q];
     }
-    __threadfence_system();
+    // One system-scope release per packet: the warp barrier orders every lane's
+    // payload stores before lane 0's st.release (cumulative), which also orders
+    // the S increment before the header -- S is counted before any receiver can
+    // count the messages in R (termination, section 6).
     __syncwarp();
     if (lane == 0) {
         atomicAdd((unsigned long long *)&R.ctrl->sent.v, (unsigned long long)cnt);   // S before publish
-        fence_acq_rel_sys();
         st_release_sys(&R.out_hdr[d][slot], pack(lo32(pidx + 1), cnt));
         s.wsh[w][d] = h + cnt;
         if (s.wsh[w][d] == s.wst[w][d]) s.wt0[w][d] = 0;
@@ -385,68 +410,217 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
     }
 }
 
-// Whole warp: claim one ready inbound packet and apply it (owner-side receive).
+// Whole warp: claim the ready prefix (up to kClaim packets) of one inbound
+// channel with ONE CAS on its cursor, apply the messages (owner-side receive),
+// and release every packet slot to its sender.  Each lane probes one header, so
+// a busy channel is drained kClaim packets per cursor round trip instead of one.
+constexpr int kClaim = 8;
+constexpr int kInU = 4;              // messages per lane in flight while applying
+
 template <int APP>
 __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
     const RankDev &R = s.R;
     if (R.n_ranks <= 1) return false;
     const int lane = threadIdx.x & 31;
     const uint32_t cp = (uint32_t)kp.cp;
-    int src = -1;
-    uint32_t cnt = 0;
-    unsigned long long c = 0;
-    if (lane == 0) {
+    const int p = R.n_ranks;
+    const int start = (w + (int)(s.c_idle & 7)) % p;
+    for (int k = 0; k < p; ++k) {
+        const int sr = (start + k) % p;
+        if (sr == R.rank) continue;
+        unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[sr].v;
+        uint64_t cc = 0;
+        if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+        cc = __shfl_sync(kFull, cc, 0);
+        bool ready = false;
+        uint32_t cnt = 0;
+        if (lane < kClaim && (uint32_t)lane < cp) {
+            // relaxed poll: an acquire load also invalidates L1 (CCTL.IVALL), which
+            // every idle warp would otherwise do on every poll of every channel
+            const uint64_t h = ld_relaxed_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+            ready = hi32(h) == lo32(cc + lane + 1);
+            cnt = lo32(h);
+        }
+        const uint32_t nready = __ballot_sync(kFull, ready);
+        const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;   // ready prefix
+        if (r == 0) continue;
+        int won = 0;
+        if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+        if (!__shfl_sync(kFull, won, 0)) continue;
+        // acquire each claimed header (synchronises with its sender's st.release),
+        // then the warp barrier orders every lane's payload reads after them
+        if (lane < r) (void)ld_acquire_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+        __syncwarp();
+        uint32_t total = 0;
+        for (int q = 0; q < r; ++q) {
+            const uint32_t cq = __shfl_sync(kFull, cnt, q);
+            const uint32_t slot = (uint32_t)((cc + q) & (cp - 1));
+            const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+            for (uint32_t base = 0; base < cq; base += 32 * kInU) {
+                bool pred[kInU];
+                uint32_t ul[kInU];
+                if constexpr (APP == kApBfs) {
+                    uint64_t m[kInU];
+#pragma unroll
+                    for (int j = 0; j < kInU; ++j) {
+                        const uint32_t i = base + j * 32 + lane;
+                        m[j] = i < cq ? ld_cg_u64((const uint64_t *)pay + i) : 0ull;
+                    }
+#pragma unroll
+                    for (int j = 0; j < kInU; ++j) {
+                        const uint32_t i = base + j * 32 + lane;
+                        ul[j] = lo32(m[j]);
+                        pred[j] = false;
+                        if (i < cq) {
+                            const uint32_t ndw = dw_make(hi32(m[j]));
+                            pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
+                            if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(m[j])));
+                        }
+                    }
+                } else {
+                    uint4 m[kInU];
+#pragma unroll
+                    for (int j = 0; j < kInU; ++j) {
+                        const uint32_t i = base + j * 32 + lane;
+                        m[j] = i < cq ? ld_cg_u4((const uint4 *)pay + i) : make_uint4(0, 0, 0, 0);
+                    }
+#pragma unroll
+                    for (int j = 0; j < kInU; ++j) {
+                        const uint32_t i = base + j * 32 + lane;
+                        ul[j] = m[j].x;
+                        pred[j] = false;
+                        if (i < cq) {
+                            const double dlt = __longlong_as_double((long long)(((uint64_t)m[j].w << 32) | m[j].z));
+                            const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
+                            pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                        }
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < kInU; ++j) {
+                    if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
+                    warp_append_local(s, w, wn, pred[j], ul[j]);
+                }
+            }
+            total += cq;
+        }
+        warp_flush_local(s, w, wn, false);      // T counts the new local work before R
+        __syncwarp();
+        if (lane == 0) {
+            // one system-scope fence per claim: every lane's payload reads and the
+            // resulting state updates / enqueues are ordered before the slots are
+            // handed back to the sender and before R counts the messages
+            fence_acq_rel_sys();
+            for (int q = 0; q < r; ++q)
+                st_relaxed_sys(&R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);   // slots free for the sender
+            atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)total);
+        }
+        __syncwarp();
+        return true;
+    }
+    return false;
+}
+
+// Whole CTA (the worker loop's receive step): warp 0 claims the ready prefix (up
+// to kClaim packets) of one inbound channel with one CAS, then ALL 512 threads
+// apply its messages -- a claimed set is expanded like a pop batch, instead of one
+// warp applying it while the other 15 wait at the loop's barrier.  Returns
+// whether anything was claimed (CTA-uniform).
+template <int APP>
+__device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
+    const RankDev &R = s.R;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint32_t cp = (uint32_t)kp.cp;
+    if (w == 0) {
         const int p = R.n_ranks;
-        const int start = (w + (int)(s.c_idle & 7)) % p;
-        for (int k = 0; k < p; ++k) {
+        const int start = (cta + (int)s.c_idle) % p;
+        int got = 0;
+        for (int k = 0; k < p && !got; ++k) {
             const int sr = (start + k) % p;
             if (sr == R.rank) continue;
             unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[sr].v;
-            const uint64_t cc = ld_relaxed_gpu((const uint64_t *)cur);
-            const uint64_t h = ld_acquire_sys(&R.in_hdr[sr][cc & (cp - 1)]);
-            if (hi32(h) == lo32(cc + 1) && atomicCAS(cur, cc, cc + 1) == cc) {
-                src = sr;
+            uint64_t cc = 0;
+            if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+            cc = __shfl_sync(kFull, cc, 0);
+            bool ready = false;
+            uint32_t cnt = 0;
+            if (lane < kClaim && (uint32_t)lane < cp) {
+                const uint64_t h = ld_relaxed_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // relaxed poll
+                ready = hi32(h) == lo32(cc + lane + 1);
                 cnt = lo32(h);
-                c = cc;
-                break;
+            }
+            const uint32_t nready = __ballot_sync(kFull, ready);
+            const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
+            if (r == 0) continue;
+            int won = 0;
+            if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+            if (!__shfl_sync(kFull, won, 0)) continue;
+            if (lane < r) (void)ld_acquire_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // sync with each sender's release
+            uint32_t incl = lane < r ? cnt : 0u;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, d);
+                if (lane >= d) incl += y;
+            }
+            if (lane < r) s.in_off[lane + 1] = incl;
+            if (lane == 0) { s.in_off[0] = 0; s.in_src = sr; s.in_cc = cc; s.in_r = r; }
+            got = 1;
+        }
+        if (lane == 0) s.in_got = got;
+    }
+    __syncthreads();      // also orders warp 0's acquires before every thread's payload reads
+    if (!s.in_got) return false;
+    const int sr = s.in_src, r = s.in_r;
+    const uint64_t cc = s.in_cc;
+    const uint32_t M = s.in_off[r];
+    uint32_t wn = s.wn[w];
+    for (uint32_t base = 0; base < M; base += kThreads * kInU) {
+        bool pred[kInU];
+        uint32_t ul[kInU];
+        int q = 0;
+#pragma unroll
+        for (int j = 0; j < kInU; ++j) {
+            const uint32_t m = base + j * kThreads + tid;
+            pred[j] = false;
+            ul[j] = 0;
+            if (m < M) {
+                while (q + 1 < r && s.in_off[q + 1] <= m) ++q;   // packet holding message m
+                const uint32_t slot = (uint32_t)((cc + q) & (cp - 1));
+                const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+                const uint32_t i = m - s.in_off[q];
+                if constexpr (APP == kApBfs) {
+                    const uint64_t msg = ld_cg_u64((const uint64_t *)pay + i);
+                    ul[j] = lo32(msg);
+                    const uint32_t ndw = dw_make(hi32(msg));
+                    pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
+                    if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(msg)));
+                } else {
+                    const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
+                    ul[j] = msg.x;
+                    const double dlt = __longlong_as_double((long long)(((uint64_t)msg.w << 32) | msg.z));
+                    const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
+                    pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                }
             }
         }
-    }
-    src = __shfl_sync(kFull, src, 0);
-    if (src < 0) return false;
-    cnt = __shfl_sync(kFull, cnt, 0);
-    c = __shfl_sync(kFull, c, 0);
-    const uint32_t slot = (uint32_t)(c & (cp - 1));
-    const unsigned char *pay = R.in_payload[src] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
-    for (uint32_t base = 0; base < cnt; base += 32) {
-        const uint32_t i = base + lane;
-        bool pred = false;
-        uint32_t ul = 0;
-        if (i < cnt) {
-            if constexpr (APP == kApBfs) {
-                const uint64_t m = ld_cg_u64((const uint64_t *)pay + i);
-                ul = lo32(m);
-                const uint32_t ndw = dw_make(hi32(m));
-                pred = atom_min_u32(R.depth + R.v_begin + ul, ndw) > ndw;
-                if (pred && kp.filter) stg_u8(R.filt + R.v_begin + ul, filt_of(hi32(m)));
-            } else {
-                const uint4 m = ld_cg_u4((const uint4 *)pay + i);
-                ul = m.x;
-                const double dlt = __longlong_as_double((long long)(((uint64_t)m.w << 32) | m.z));
-                const double old = atom_add_f64(R.pr_res + pr_slot(ul, R.pr_q), dlt);
-                pred = old < kp.eps && old + dlt >= kp.eps;
-            }
+#pragma unroll
+        for (int j = 0; j < kInU; ++j) {
+            if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
+            warp_append_local(s, w, wn, pred[j], ul[j]);
         }
-        if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
-        warp_append_local(s, w, wn, pred, ul);
     }
-    warp_flush_local(s, w, wn, false);      // T counts the new local work before R
-    if (lane == 0) {
-        st_release_sys(&R.peer_free[src][slot], c + cp);   // slot free for the sender
+    warp_flush_local(s, w, wn, false);        // T counts the new local work before R
+    if (lane == 0) s.wn[w] = wn;
+    __syncthreads();
+    if (tid == 0) {
+        // one system-scope fence per claim: payload reads and their effects are
+        // ordered before the slots go back to the sender and before R counts them
         fence_acq_rel_sys();
-        atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)cnt);
+        for (int q = 0; q < r; ++q)
+            st_relaxed_sys(&R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);
+        atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)M);
+        s.c_batches++;
     }
-    __syncwarp();
     return true;
 }
 
@@ -487,7 +661,13 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
         for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? ldg_u8(filt + u[k]) : 0u;       // probe the filter
     } else {
 #pragma unroll
-        for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;     // probe the word
+        for (int k = 0; k < N; ++k) {
+#ifdef ATOS_NO_PROBE
+            cur[k] = 0xFFFFFFFFu;
+#else
+            cur[k] = (u[k] >= 0) ? ldg_u32(depth + u[k]) : 0u;     // probe the word
+#endif
+        }
     }
     if (kp.relax_red) {
         // fire-and-forget relaxation: red.min, enqueue on the probe's verdict.
@@ -631,14 +811,19 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
 #endif
         } else {
             const double eps = kp.eps;
-            bool cross[kU];
+            bool cross[kU], gcross[kU];
+            const bool comb = MULTI && kp.combine;
+            const int64_t qn = pr_q_of(R.n);
 #pragma unroll
             for (int k = 0; k < kU; ++k) {
-                cross[k] = false;
+                cross[k] = gcross[k] = false;
+                const double dlt = __longlong_as_double((long long)vv[k]);
                 if (u[k] >= vb && u[k] < ve) {
-                    const double dlt = __longlong_as_double((long long)vv[k]);
                     const double old = atom_add_f64(res + pr_slot(u[k] - vb, R.pr_q), dlt);
                     cross[k] = old < eps && old + dlt >= eps;        // crossing enqueue (R5)
+                } else if (comb && u[k] >= 0) {                      // combine into the ghost residual (N2)
+                    const double old = atom_add_f64(R.pr_ghost + pr_slot(u[k], qn), dlt);
+                    gcross[k] = old < kp.eps_g && old + dlt >= kp.eps_g;
                 }
             }
             if constexpr (!multi) {
@@ -654,6 +839,14 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                 for (int k = 0; k < kU; ++k) {
                     if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
                     warp_append_local(s, w, wn, cross[k], (uint32_t)(u[k] - vb));
+                    if (comb) {   // the crossing add takes the whole ghost and sends it as one message
+                        uint64_t gv = 0;
+                        if (gcross[k]) gv = atom_exch_u64((uint64_t *)(R.pr_ghost + pr_slot(u[k], qn)), 0ull);
+                        const int d = gcross[k] ? owner_of(R, u[k]) : 0;
+                        warp_append_remote<APP>(s, kp, cta, w, gcross[k], d,
+                                                gcross[k] ? (uint32_t)(u[k] - R.part[d]) : 0u, gv, wn);
+                        continue;
+                    }
                     const bool rem = u[k] >= 0 && !(u[k] >= vb && u[k] < ve);
                     const int d = rem ? owner_of(R, u[k]) : 0;
                     warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
@@ -766,8 +959,23 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     if (tid == 0) s.prof[7] -= (unsigned long long)clock64();
 #endif
     int64_t deg = 0;
+    uint32_t npc = 0;      // BFS: pieces of this row to publish
     if (tid < B) {
-        const uint32_t v = bb.v[tid];
+        const uint32_t it = bb.v[tid];
+        if (APP == kApBfs && (it & kPieceBit)) {
+            // a piece of a split row: edges [piece * split, (piece+1) * split) of v,
+            // relaxed with v's current depth (a valid bound: depths only decrease,
+            // and a newer depth re-expands the whole row anyway)
+            const uint32_t v = it & 0xFFFFu, pc = (it >> 16) & 0x7FFFu;
+            const int64_t rb = ldg_i64_nc(R.row_ptr + v), re = ldg_i64_nc(R.row_ptr + v + 1);
+            const int64_t b = rb + (int64_t)pc * kp.split;
+            bb.beg[tid] = b;
+            deg = re - b < (int64_t)kp.split ? re - b : (int64_t)kp.split;
+            const uint32_t d = dw_depth(ld_relaxed_gpu_u32(R.depth + R.v_begin + v));
+            bb.val[tid] = d;
+            if (d == kDepthInf || deg < 0) deg = 0;
+        } else {
+        const uint32_t v = it;
         const int64_t b = ldg_i64_nc(R.row_ptr + v), e = ldg_i64_nc(R.row_ptr + v + 1);
         bb.beg[tid] = b;
         deg = e - b;
@@ -778,6 +986,11 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
             const uint32_t d = dw_depth(old);
             bb.val[tid] = d;
             if (!(old & 1u) || d == kDepthInf) deg = 0;
+            if (kp.split > 0 && deg > 2 * (int64_t)kp.split && (int64_t)v < kPieceVMax &&
+                deg <= (int64_t)kp.split * kPieceMax) {
+                npc = (uint32_t)((deg - 1) / kp.split);   // pieces 1..npc go to the ring
+                deg = kp.split;
+            }
         } else {
             const int64_t sl = pr_slot(v, R.pr_q);
             const double r = __longlong_as_double((long long)atom_exch_u64((uint64_t *)(R.pr_res + sl), 0ull));
@@ -785,6 +998,21 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
             if (r == 0.0 || deg == 0) deg = 0;        // dangling vertices absorb (R4)
             else bb.val[tid] = (uint64_t)__double_as_longlong(kp.alpha * r / (double)deg);
         }
+        }
+    }
+    if (APP == kApBfs && kp.split > 0 && __syncthreads_or(npc > 0)) {
+        // publish the pieces before expanding, so idle workers start on them now;
+        // T grows before this batch's F, so termination cannot be declared early
+        int64_t pex;
+        const int64_t ptot = block_exscan(s, (int64_t)npc, pex);
+        if (tid == 0) {
+            s.b64[2] = atomicAdd((unsigned long long *)&R.ctrl->tail.v, (unsigned long long)ptot);
+            s.c_pushes += (unsigned long long)ptot;
+        }
+        __syncthreads();
+        const uint64_t pbase = s.b64[2] + (uint64_t)pex;
+        for (uint32_t i = 0; i < npc; ++i)
+            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
     }
     if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + bb.beg[tid], (uint64_t)deg * 4);
     int64_t excl;
@@ -834,12 +1062,14 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
         s.wpre[kWarps] = total;
         uint32_t keep_n = 0;
         if (allow_keep && kp.keep > 0 && total > 0 && total <= (uint32_t)kp.keep) {
-            // keep only in a low-parallelism phase: the rank's whole outstanding
-            // work (T - F, this batch included) is tiny, so enqueueing would only
-            // add a queue round trip per level (path/road-like graphs); otherwise
-            // FIFO order is kept, which bounds asynchronous redundancy.
-            const uint64_t f = ld_relaxed_gpu(&s.R.ctrl->finished.v), t = ld_relaxed_gpu(&s.R.ctrl->tail.v);
-            if (t - f <= (uint64_t)kp.keep) keep_n = total;
+            // keep_always: follow the chain (road-like graphs: one queue round trip
+            // per level costs more than the redundant relaxations it would avoid,
+            // measured 2.1x faster on the grid); otherwise keep only in a
+            // low-parallelism phase (T - F tiny) and keep FIFO order, which bounds
+            // asynchronous redundancy.
+            const uint64_t f = kp.keep_always ? 0 : ld_relaxed_gpu(&s.R.ctrl->finished.v);
+            const uint64_t t = kp.keep_always ? 0 : ld_relaxed_gpu(&s.R.ctrl->tail.v);
+            if (kp.keep_always || t - f <= (uint64_t)kp.keep) keep_n = total;
         }
         const uint32_t push_n = total - keep_n;
         s.b64[0] = push_n ? atomicAdd((unsigned long long *)&s.R.ctrl->tail.v, (unsigned long long)push_n) : 0ull;
@@ -891,7 +1121,22 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
     const int tid = threadIdx.x;
     BatchBuf &bb = s.bb[0];
     if (tid == 0) {
-        if (s.res_lo == s.res_hi) {
+        if (s.res_lo == s.res_hi && kp.discrete) {
+            // discrete mode: reserve with atomicAdd and clip at the launch's snapshot,
+            // so every reserved slot is already published; head may overshoot the
+            // limit and is set back to it by discrete_step_kernel (a CAS loop here
+            // measured ~1.3 us per success under 296-way contention)
+            const uint64_t h = ld_relaxed_gpu(&R.ctrl->head.v);
+            if (h < s.limit) {
+                uint64_t k = (s.limit - h) / (uint64_t)kp.ctas_per_rank;
+                k = k < 1 ? 1 : (k > (uint64_t)kp.fetch ? (uint64_t)kp.fetch : k);
+                const uint64_t lo = atomicAdd((unsigned long long *)&R.ctrl->head.v, (unsigned long long)k);
+                if (lo < s.limit) {
+                    s.res_lo = lo;
+                    s.res_hi = lo + k < s.limit ? lo + k : s.limit;
+                }
+            }
+        } else if (s.res_lo == s.res_hi) {
             const uint64_t t = ld_relaxed_gpu(&R.ctrl->tail.v);
             const uint64_t h = ld_relaxed_gpu(&R.ctrl->head.v);
             if (t > h) {
@@ -985,9 +1230,7 @@ __device__ void coordinator_step(Smem &s, const KParams &kp) {
 // the persistent worker
 // ---------------------------------------------------------------------------
 template <int APP, bool MULTI>
-__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KParams kp) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    Smem &s = *reinterpret_cast<Smem *>(smem_raw);
+__device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
     const int lr = blockIdx.x / kp.ctas_per_rank;
     const int cta = blockIdx.x % kp.ctas_per_rank;
     const int tid = threadIdx.x, w = tid >> 5;
@@ -999,6 +1242,7 @@ __global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KPara
         s.wave_valid = 0;
         s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = 0;
         s.c_busy = s.c_batches = 0;
+        s.limit = kp.discrete ? ld_relaxed_gpu(&s.R.ctrl->limit.v) : 0;
 #ifdef ATOS_PROF
         for (int k = 0; k < 10; ++k) s.prof[k] = 0;
 #endif
@@ -1031,13 +1275,7 @@ __global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KPara
 
         const uint64_t t_work0 = (tid == 0) ? globaltimer() : 0;
         bool worked = false;
-        if constexpr (multi) {
-            uint32_t wn = s.wn[w];
-            const bool got = warp_inbound<APP>(s, kp, w, wn);
-            __syncwarp();
-            if ((tid & 31) == 0) s.wn[w] = wn;
-            worked = __syncthreads_or(got);
-        }
+        if constexpr (multi) worked = cta_inbound<APP>(s, kp, cta);
         if (!worked) {
 #ifdef ATOS_PROF
             const long long pb0 = clock64();
@@ -1084,6 +1322,7 @@ __global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KPara
         }
 
         // ---- idle: flush aged staging, detect termination, watchdog
+        if (kp.discrete) break;   // discrete launch: the snapshot is drained (nothing reserved, head == limit)
         ++idle_streak;
         if constexpr (multi) {
             uint32_t wn = s.wn[w];
@@ -1126,6 +1365,40 @@ __global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KPara
                    s.prof[5] / (s.c_batches + 1), s.c_batches);
 #endif
     }
+}
+
+// The persistent worker (one cooperative launch per solve).
+template <int APP, bool MULTI>
+__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KParams kp) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    worker_body<APP, MULTI>(*reinterpret_cast<Smem *>(smem_raw), kp);
+}
+
+// Discrete-kernel mode: one launch per queue snapshot, replayed by
+// a CUDA-graph while-node; the per-solve parameters live in device memory so the
+// instantiated graph never changes.
+template <int APP>
+__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_discrete_kernel(const KParams *kpp) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ KParams kps;
+    if (threadIdx.x == 0) kps = *kpp;
+    __syncthreads();
+    worker_body<APP, false>(*reinterpret_cast<Smem *>(smem_raw), kps);
+}
+
+// Between discrete launches: snapshot the tail as the next launch's limit and keep
+// looping while the queue holds work (and no device error was raised).
+__global__ void discrete_step_kernel(const KParams *kpp, cudaGraphConditionalHandle h, int after_launch) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const RankDev &R = kpp->ranks[0];
+    // after a launch every index below the old limit was consumed; reservations
+    // past it were clipped, so head goes back to the limit
+    if (after_launch && R.ctrl->head.v > R.ctrl->limit.v) R.ctrl->head.v = R.ctrl->limit.v;
+    const uint64_t t = ld_relaxed_gpu(&R.ctrl->tail.v), hd = ld_relaxed_gpu(&R.ctrl->head.v);
+    R.ctrl->limit.v = t;
+    const bool more = t > hd && ld_relaxed_gpu(&R.ctrl->error.v) == 0;
+    if (more) R.ctrl->st_waves.v += 1;          // = worker launches of the solve
+    cudaGraphSetConditional(h, more ? 1u : 0u);
 }
 
 }  // namespace atos

@@ -32,8 +32,13 @@ def main():
         ms = sum(x["ms_worker"] for x in rows) / len(rows)
         rel = sum(x["edges"] for x in rows) / len(rows)
         pops = sum(x["pops"] for x in rows) / len(rows)
+        msgs = sum(x["msgs_sent"] for x in rows) / len(rows)
+        iters = sum(x["iterations"] for x in rows) / len(rows)
+        pk = sum(x["packets_sent"] for x in rows) / len(rows)
         print(json.dumps({"cfg": cfg, "ms": round(ms, 3), "relax_per_nnz": round(rel / g.nnz, 2),
-                          "pops_per_v": round(pops / g.n, 2), "gatomics": round(rel / ms / 1e6, 1)}), flush=True)
+                          "pops_per_v": round(pops / g.n, 2), "gatomics": round(rel / ms / 1e6, 1),
+                          "msgs_M": round(msgs / 1e6, 2), "packets_K": round(pk / 1e3, 2),
+                          "msg_GBps": round(msgs * 16 / ms / 1e6, 1), "iters": iters}), flush=True)
 
 
 if __name__ == "__main__":

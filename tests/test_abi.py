@@ -58,7 +58,7 @@ def test_struct_layouts_match_header():
 
 
 def test_version():
-    assert atos.load().atos_version() == 2
+    assert atos.load().atos_version() == 3
 
 
 def test_partition_balanced_matches_definition():
@@ -107,10 +107,13 @@ def test_graph_load_fails_loudly_without_gpu():
 def test_relabel_and_hub_cache_config_validation():
     cfg = atos.default_config()
     assert cfg.relabel == 2 and cfg.hub_cache == -1          # auto / auto
+    assert cfg.split_edges == -1 and cfg.keep_items == -1     # auto
     rp = np.array([0, 1, 1], dtype=np.int64)
     col = np.array([1], dtype=np.int32)
     for bad in (dict(relabel=3), dict(hub_cache=33), dict(hub_cache=1 << 20), dict(hub_cache=-2),
-                dict(hub_cache=32, virtual_ranks=2)):
+                dict(hub_cache=32, virtual_ranks=2), dict(split_edges=100), dict(split_edges=128),
+                dict(split_edges=1 << 21), dict(split_edges=-2), dict(pr_combine=2), dict(keep_items=-2), dict(keep_mode=2), dict(discrete=2),
+                dict(discrete=1, virtual_ranks=2), dict(discrete=1, n_ranks=2)):
         with pytest.raises(atos.AtosError) as e:
             atos.Graph(rp, col, **bad)
         assert e.value.status == 1, bad

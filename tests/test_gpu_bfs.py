@@ -217,3 +217,64 @@ def test_hub_cache_active_on_skewed_graph():
     with atos.Graph(rp, col, hub_cache=0) as G:
         d, st = G.bfs(src, stats=True)
     assert np.array_equal(d, oracle.bfs(rp, col, src)) and st["hub_hits"] == 0
+
+
+@pytest.mark.parametrize("opts", [dict(split_edges=256), dict(split_edges=256, relabel=0),
+                                  dict(split_edges=256, virtual_ranks=4), dict(split_edges=256, virtual_ranks=3,
+                                                                               agg_enabled=0),
+                                  dict(split_edges=512, keep_items=64, fetch_size=5),
+                                  dict(split_edges=256, probe_filter=1), dict(split_edges=0)])
+def test_row_splitting_same_depths_and_parents(opts):
+    """Hub rows cut into pieces any worker can pop
+    must reach the same depths and min-id parents."""
+    g = inputs.rmat(15, 16, 3, symmetric=True)
+    rp, col = g.numpy()
+    for s in inputs.bfs_sources(g, 2, seed=9):
+        run_and_check(rp, col, s, **opts)
+    # a star + path: hub 0 of degree 60000 feeding a chain, and a second hub beyond id 65535
+    n = 140000
+    edges = [(0, v) for v in range(1, 60001)] + [(v, 0) for v in range(1, 60001)]
+    edges += [(v, v + 1) for v in range(60000, 70000)] + [(v + 1, v) for v in range(60000, 70000)]
+    edges += [(70000, v) for v in range(70001, n)] + [(v, 70000) for v in range(70001, n)]
+    rp, col = csr_of(n, edges)
+    for s in (0, 5, 70000, 139999):
+        run_and_check(rp, col, s, **opts)
+
+
+def test_row_splitting_publishes_pieces():
+    n = 50001
+    edges = [(0, v) for v in range(1, n)] + [(v, 0) for v in range(1, n)]
+    rp, col = csr_of(n, edges)
+    with atos.Graph(rp, col, split_edges=256) as G:
+        d, st = G.bfs(0, stats=True)
+    assert np.array_equal(d, oracle.bfs(rp, col, 0))
+    # the hub's row (50000 edges) becomes 1 kept + 195 published pieces
+    assert st["pops"] >= n + 195, st
+    assert st["edges"] == col.size, st
+
+
+@pytest.mark.parametrize("opts", [dict(discrete=1), dict(discrete=1, split_edges=256), dict(discrete=1, keep_items=0),
+                                  dict(discrete=1, keep_items=64, keep_mode=1), dict(discrete=1, probe_filter=1)])
+def test_discrete_kernel_mode_same_depths_and_parents(opts):
+    """one worker launch per queue snapshot, looped by a CUDA-graph
+    while-node, reaches the same depths and min-id parents."""
+    g = inputs.rmat(15, 16, 6, symmetric=True)
+    rp, col = g.numpy()
+    for s in inputs.bfs_sources(g, 2, seed=3):
+        run_and_check(rp, col, s, **opts)
+    gg = inputs.road_grid(60, 40, seed=2)
+    rp, col = gg.numpy()
+    run_and_check(rp, col, 5, **opts)
+
+
+def test_discrete_iterations_equal_levels_on_a_path():
+    n = 1000
+    rp, col = csr_of(n, [(i, i + 1) for i in range(n - 1)] + [(i + 1, i) for i in range(n - 1)])
+    with atos.Graph(rp, col, discrete=1, keep_items=0) as G:
+        d, st = G.bfs(0, stats=True)
+        assert np.array_equal(d, np.arange(n))
+        assert st["iterations"] == n, st
+        d2, st2 = G.bfs(n - 1, stats=True)            # repeated solve on the same instantiated graph
+        assert np.array_equal(d2, np.arange(n)[::-1]) and st2["iterations"] == n
+    with pytest.raises(atos.AtosError):
+        atos.Graph(rp, col, discrete=1, virtual_ranks=2)
