@@ -732,7 +732,11 @@ static KParams make_params(atos_graph *g) {
     kp.cp = g->S.cp;
     kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
-    kp.keep = g->cfg.keep_items >= 0 ? g->cfg.keep_items : (g->skewed ? 0 : kKeepAuto);
+    // auto keeping: only for a persistent single-rank solve on a non-skewed graph
+    // (discrete launches chain without bound inside one launch: 87 edges per
+    // m_reached on the grid; measured)
+    kp.keep = g->cfg.keep_items >= 0 ? g->cfg.keep_items
+                                     : ((g->skewed || g->cfg.discrete || g->p > 1) ? 0 : kKeepAuto);
     kp.keep_always = g->cfg.keep_items >= 0 ? g->cfg.keep_mode : 1;
     kp.prefetch = g->cfg.prefetch;
     kp.relax_red = g->cfg.relax_red;
@@ -744,6 +748,7 @@ static KParams make_params(atos_graph *g) {
     kp.hc_per_rank = g->hc_per_rank;
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
+    kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;

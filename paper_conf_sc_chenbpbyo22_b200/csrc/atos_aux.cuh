@@ -12,13 +12,13 @@ __global__ void barrier_kernel(KParams kp, uint64_t value) {
     if (threadIdx.x != 0) return;
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
-        for (int d = 0; d < R.n_ranks; ++d) st_release_sys(&R.peer_ctrl[d]->bar[R.rank].v, value);
+        for (int d = 0; d < R.n_ranks; ++d) st_release_peer(kp.sys, &R.peer_ctrl[d]->bar[R.rank].v, value);
     }
     const uint64_t t0 = globaltimer();
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         for (int d = 0; d < R.n_ranks; ++d) {
-            while (ld_acquire_sys(&R.ctrl->bar[d].v) < value) {
+            while (ld_acquire_peer(kp.sys, &R.ctrl->bar[d].v) < value) {
                 if (kp.watchdog_ns > 0 && globaltimer() - t0 > (uint64_t)kp.watchdog_ns) {
                     set_error(R, kErrTimeout);
                     return;

@@ -95,6 +95,26 @@ __device__ __forceinline__ uint64_t globaltimer() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// Peer-visible accesses at the scope the peers need: other GPUs / processes need
+// .sys; virtual ranks (all peers on this device) need only .gpu, whose fences do
+// not drain to the system level (MEMBAR.GPU instead of MEMBAR.SYS).  `sys` is
+// uniform per launch (KParams::sys).
+__device__ __forceinline__ uint64_t ld_acquire_peer(bool sys, const uint64_t *p) {
+    return sys ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+}
+__device__ __forceinline__ uint64_t ld_relaxed_peer(bool sys, const uint64_t *p) {
+    return sys ? ld_relaxed_sys(p) : ld_relaxed_gpu(p);
+}
+__device__ __forceinline__ void st_release_peer(bool sys, uint64_t *p, uint64_t v) {
+    if (sys) st_release_sys(p, v); else st_release_gpu(p, v);
+}
+__device__ __forceinline__ void st_relaxed_peer(bool sys, uint64_t *p, uint64_t v) {
+    if (sys) st_relaxed_sys(p, v); else st_relaxed_gpu(p, v);
+}
+__device__ __forceinline__ void fence_peer(bool sys) {
+    if (sys) fence_acq_rel_sys(); else fence_acq_rel_gpu();
+}
+
 // Explicit global-space accesses.  The rank view lives in shared memory, so the
 // compiler cannot prove its pointers are global and would emit generic LD/ATOM;
 // these force LDG / ATOMG without a "memory" clobber (no forced smem reloads).
@@ -249,6 +269,7 @@ struct KParams {
     int32_t split;           // BFS row pieces: edges per piece (0 = off), see kPieceBit
     int32_t combine;         // PR sender-side residual combining (multi-rank)
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained
+    int32_t sys;             // peers are other devices/processes: system-scope ordering (else .gpu)
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

@@ -309,7 +309,7 @@ __device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int
     for (;;) {   // wait for the receiver to free the slot; keep consuming inbound meanwhile
         int st = 0;
         if (lane == 0) {
-            const uint64_t f = ld_acquire_sys(&R.free_mirror[d][slot]);
+            const uint64_t f = ld_acquire_peer(kp.sys, &R.free_mirror[d][slot]);
             if (lo32(f) == lo32(pidx)) st = 1;
             else {
                 const uint64_t now = globaltimer();
@@ -341,7 +341,7 @@ __device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int
     __syncwarp();
     if (lane == 0) {
         atomicAdd((unsigned long long *)&R.ctrl->sent.v, (unsigned long long)cnt);   // S before publish
-        st_release_sys(&R.out_hdr[d][slot], pack(lo32(pidx + 1), cnt));
+        st_release_peer(kp.sys, &R.out_hdr[d][slot], pack(lo32(pidx + 1), cnt));
         s.wsh[w][d] = h + cnt;
         if (s.wsh[w][d] == s.wst[w][d]) s.wt0[w][d] = 0;
         atomicAdd(&s.c_msgs, (unsigned long long)cnt);
@@ -437,7 +437,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
         if (lane < kClaim && (uint32_t)lane < cp) {
             // relaxed poll: an acquire load also invalidates L1 (CCTL.IVALL), which
             // every idle warp would otherwise do on every poll of every channel
-            const uint64_t h = ld_relaxed_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+            const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);
             ready = hi32(h) == lo32(cc + lane + 1);
             cnt = lo32(h);
         }
@@ -449,7 +449,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
         if (!__shfl_sync(kFull, won, 0)) continue;
         // acquire each claimed header (synchronises with its sender's st.release),
         // then the warp barrier orders every lane's payload reads after them
-        if (lane < r) (void)ld_acquire_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+        if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);
         __syncwarp();
         uint32_t total = 0;
         for (int q = 0; q < r; ++q) {
@@ -510,9 +510,9 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
             // one system-scope fence per claim: every lane's payload reads and the
             // resulting state updates / enqueues are ordered before the slots are
             // handed back to the sender and before R counts the messages
-            fence_acq_rel_sys();
+            fence_peer(kp.sys);
             for (int q = 0; q < r; ++q)
-                st_relaxed_sys(&R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);   // slots free for the sender
+                st_relaxed_peer(kp.sys, &R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);   // slots free for the sender
             atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)total);
         }
         __syncwarp();
@@ -545,7 +545,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
             bool ready = false;
             uint32_t cnt = 0;
             if (lane < kClaim && (uint32_t)lane < cp) {
-                const uint64_t h = ld_relaxed_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // relaxed poll
+                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // relaxed poll
                 ready = hi32(h) == lo32(cc + lane + 1);
                 cnt = lo32(h);
             }
@@ -555,7 +555,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
             int won = 0;
             if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
             if (!__shfl_sync(kFull, won, 0)) continue;
-            if (lane < r) (void)ld_acquire_sys(&R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // sync with each sender's release
+            if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // sync with each sender's release
             uint32_t incl = lane < r ? cnt : 0u;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
@@ -615,9 +615,9 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
     if (tid == 0) {
         // one system-scope fence per claim: payload reads and their effects are
         // ordered before the slots go back to the sender and before R counts them
-        fence_acq_rel_sys();
+        fence_peer(kp.sys);
         for (int q = 0; q < r; ++q)
-            st_relaxed_sys(&R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);
+            st_relaxed_peer(kp.sys, &R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);
         atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)M);
         s.c_batches++;
     }
@@ -1096,7 +1096,7 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
 }
 
 // Report this CTA's staged-message count change to the rank counter.
-__device__ void report_staged(Smem &s) {
+__device__ void report_staged(Smem &s, const KParams &kp) {
     if (s.R.n_ranks <= 1) return;
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -1105,7 +1105,7 @@ __device__ void report_staged(Smem &s) {
             for (int d = 0; d < s.R.n_ranks; ++d) cur += (uint64_t)(s.wst[w][d] - s.wsh[w][d]);
         const uint64_t delta = cur - s.staged_reported;   // mod 2^64
         if (delta != 0) {
-            fence_acq_rel_sys();
+            fence_peer(kp.sys);
             atomicAdd((unsigned long long *)&s.R.ctrl->staged.v, (unsigned long long)delta);
             s.staged_reported = cur;
         }
@@ -1186,13 +1186,13 @@ __device__ void coordinator_step(Smem &s, const KParams &kp) {
     bool started = true;
     uint64_t F = 0, Rv = 0, T = 0, St = 0, S = 0;
     if (lane < p) {
-        started = ld_acquire_sys(&R.ctrl->started[lane].v) == kp.epoch;
+        started = ld_acquire_peer(kp.sys, &R.ctrl->started[lane].v) == kp.epoch;
         const Ctrl *c = R.peer_ctrl[lane];
-        F = ld_acquire_sys(&c->finished.v);
-        Rv = ld_acquire_sys(&c->recvd.v);
-        T = ld_acquire_sys(&c->tail.v);
-        St = ld_acquire_sys(&c->staged.v);
-        S = ld_acquire_sys(&c->sent.v);
+        F = ld_acquire_peer(kp.sys, &c->finished.v);
+        Rv = ld_acquire_peer(kp.sys, &c->recvd.v);
+        T = ld_acquire_peer(kp.sys, &c->tail.v);
+        St = ld_acquire_peer(kp.sys, &c->staged.v);
+        S = ld_acquire_peer(kp.sys, &c->sent.v);
     }
     if (!__all_sync(kFull, started)) {
         if (lane == 0) s.wave_valid = 0;
@@ -1220,7 +1220,7 @@ __device__ void coordinator_step(Smem &s, const KParams &kp) {
     }
     if (lane == 0) s.wave_valid = all_passive && sumS == sumR;
     if (all_same && all_passive && sumS == sumR) {
-        if (lane < p) st_release_sys(&R.peer_ctrl[lane]->done.v, kp.epoch);
+        if (lane < p) st_release_peer(kp.sys, &R.peer_ctrl[lane]->done.v, kp.epoch);
     }
     if (lane == 0) atomicAdd((unsigned long long *)&R.ctrl->st_waves.v, 1ull);
     __syncwarp();
@@ -1259,7 +1259,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
     __syncthreads();
     constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
-    if (tid == 0 && cta == 0) st_release_sys(&s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
+    if (tid == 0 && cta == 0) st_release_peer(kp.sys, &s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
     const uint64_t t_start = globaltimer();
     uint32_t idle_streak = 0;
 
@@ -1301,7 +1301,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
                     if (tid == 0) s.prof[9] += (unsigned long long)(clock64() - pb2);
 #endif
                 }
-                report_staged(s);
+                report_staged(s, kp);
 #ifdef ATOS_PROF
                 if (tid == 0) { s.prof[5] += (unsigned long long)(clock64() - pb0); }
 #endif
@@ -1309,7 +1309,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
                     // T (returned by its atomic before the slot stores) is performed
                     // before this F update is issued; multi-rank adds a sys fence
                     // because the coordinator reads these counters over NVLink
-                    if (multi) fence_acq_rel_sys();
+                    if (multi) fence_peer(kp.sys);
                     atomicAdd((unsigned long long *)&s.R.ctrl->finished.v, (unsigned long long)B0);  // F last
                 }
                 worked = true;
@@ -1329,7 +1329,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
             warp_flush_remote<APP>(s, kp, cta, w, true, wn);
             warp_flush_local(s, w, wn, false);
             if ((tid & 31) == 0) s.wn[w] = wn;
-            report_staged(s);
+            report_staged(s, kp);
         }
         if (tid == 0) {
             s.c_idle++;
