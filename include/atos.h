@@ -72,7 +72,10 @@ typedef struct {
                                  skipped at pop); 0 = atomicMin with return   */
     int32_t pipeline;         /* BFS: 1 = software-pipelined expansion (each
                                  warp keeps two 128-edge chunks in flight),
-                                 2 = only for low-degree batches, 0 = never   */
+                                 2 = only for low-degree batches, 0 = never,
+                                 3 = three-stage pipeline (probes of the next
+                                 chunk and columns of the one after in flight
+                                 while a chunk is relaxed; no hub cache)      */
     int32_t probe_filter;     /* BFS: 1 = probe a 1-byte-per-vertex depth upper
                                  bound instead of the 4-byte words, 0 = never,
                                  2 = when the words exceed the L2 carve-out   */

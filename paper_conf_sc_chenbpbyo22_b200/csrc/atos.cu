@@ -180,6 +180,14 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     return L;
 }
 
+// sub-channels per channel: about 8 inbound cursors per rank in total (a single
+// cursor serialised the receive side at 2 ranks), each sub-channel >= 2 packets
+static int nsub_for(int p, int cp) {
+    int k = 1;
+    while (k < kMaxSub && k * 2 * (p - 1) <= 8 && cp / (k * 2) >= 2) k *= 2;
+    return p > 1 ? k : 1;
+}
+
 static int stage_cap_for(int pkt) { return (int)pow2_ceil((uint64_t)std::max(2 * pkt, 64)); }
 
 // ---------------------------------------------------------------------------
@@ -321,12 +329,12 @@ __global__ void check_rows_kernel(const int64_t *rp, int64_t nr, int64_t m, cons
         if (col[e] < 0 || col[e] >= n) atomicOr(bad, 2ull);
 }
 
-__global__ void init_arena_kernel(uint64_t *ring, uint64_t cap, uint64_t *free_m, uint64_t nfree, uint64_t cp) {
+__global__ void init_arena_kernel(uint64_t *ring, uint64_t cap, uint64_t *free_m, uint64_t nfree, uint64_t cps) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += stride)
         ring[i] = pack(lo32(i), 0u);   // free for the producer of index i
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nfree; i += stride)
-        free_m[i] = i % cp;            // packet slot i free for packet index i
+        free_m[i] = i % cps;           // slot of sub-channel packet index j (< cps) free for index j
 }
 
 // ---------------------------------------------------------------------------
@@ -665,7 +673,8 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         }
         const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
         init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
-                                                       (uint64_t *)(me.arena + me.L.free_m), nfree, g->S.cp);
+                                                       (uint64_t *)(me.arena + me.L.free_m), nfree,
+                                                       (uint64_t)(g->S.cp / nsub_for(g->p, g->S.cp)));
         CU(cudaGetLastError());
     }
     unsigned long long bad = 0;
@@ -730,6 +739,8 @@ static KParams make_params(atos_graph *g) {
     kp.fetch = g->cfg.fetch_size;
     kp.pkt = g->S.pkt;
     kp.cp = g->S.cp;
+    kp.nsub = nsub_for(g->p, g->S.cp);
+    kp.cps = g->S.cp / kp.nsub;
     kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
     // auto keeping: only for a persistent single-rank solve on a non-skewed graph
@@ -768,7 +779,11 @@ static bool l2_window(atos_graph *g, const KParams &kp, cudaAccessPolicyWindow &
                                : (void *)(me.arena + me.L.res);
     size_t bytes = APP == kApBfs ? (size_t)g->n * (kp.filter ? 1 : 4) : (size_t)me.L.n_r * 8;
     bytes = std::min(bytes, g->window_max);
+#ifdef ATOS_CARVE_MAX   // experiment: the whole persisting limit as carve-out
+    const size_t carve = g->persist_max;
+#else
     const size_t carve = std::min(bytes, g->persist_max);   // carve-out == window, no more
+#endif
     if (carve != g->persist_set) {
         if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve) != cudaSuccess) {
             cudaGetLastError();

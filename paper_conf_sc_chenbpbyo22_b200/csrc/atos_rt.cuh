@@ -14,6 +14,7 @@
 namespace atos {
 
 constexpr int kMaxRanks = 8;
+constexpr int kMaxSub = 8;                    // sub-channels per (source, destination) pair
 constexpr uint32_t kInf = 0xFFFFFFFFu;        // BFS word of an undiscovered vertex
 constexpr uint32_t kDepthInf = 0x7FFFFFFFu;   // its depth field
 
@@ -202,8 +203,8 @@ struct Ctrl {
     Line error;                  // DevError of the current solve
     Line started[kMaxRanks];     // [coordinator only] epoch each rank started
     Line bar[kMaxRanks];         // pre-init barrier arrivals (epoch per rank)
-    Line out_reserve[kMaxRanks]; // packets reserved on channel (this -> d)
-    Line in_cursor[kMaxRanks];   // next packet to consume on channel (s -> this)
+    Line out_reserve[kMaxRanks * kMaxSub]; // packets reserved on sub-channel (this -> d, k) at [d * nsub + k]
+    Line in_cursor[kMaxRanks * kMaxSub];   // next packet to consume on sub-channel (s -> this, k)
     Line ring_base;              // tail at the start of the current solve
     Line limit;                  // discrete mode: queue snapshot this launch may pop up to
     Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_hits, st_waves;
@@ -256,7 +257,8 @@ struct KParams {
     int32_t ctas_per_rank;
     int32_t fetch;           // vertices per pop batch (<= kThreads)
     int32_t pkt;             // messages per packet
-    int32_t cp;              // packets per channel (pow2)
+    int32_t cp;              // packets per channel (pow2) = nsub sub-channels of cps packets
+    int32_t nsub, cps;       // sub-channels per channel, packets per sub-channel (pow2)
     int32_t stage_cap;       // staging capacity per (cta, warp, dst), messages (pow2)
     int32_t agg_on;
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)

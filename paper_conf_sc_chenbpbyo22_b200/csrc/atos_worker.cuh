@@ -296,15 +296,22 @@ __device__ __forceinline__ unsigned char *wstage(const Smem &s, const KParams &k
 template <int APP> __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn);
 
 // Whole warp: publish `cnt` staged messages for dst as one packet.
+// A channel (s -> d) is nsub independent sub-channels (rings of cps packets,
+// own reserve counter and receive cursor); a sending warp always uses the same
+// one, so receivers claiming on different cursors do not serialise on one CAS.
+__device__ __forceinline__ uint32_t sub_slot(const KParams &kp, int k, uint64_t i) {
+    return (uint32_t)k * (uint32_t)kp.cps + (uint32_t)(i & (uint64_t)(kp.cps - 1));
+}
+
 template <int APP>
 __device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int d, uint32_t cnt, uint32_t &wn) {
     const RankDev &R = s.R;
     const int lane = threadIdx.x & 31;
-    const uint32_t cp = (uint32_t)kp.cp;
+    const int k = (cta * kWarps + w) % kp.nsub;
     unsigned long long pidx = 0;
-    if (lane == 0) pidx = atomicAdd((unsigned long long *)&R.ctrl->out_reserve[d].v, 1ull);
+    if (lane == 0) pidx = atomicAdd((unsigned long long *)&R.ctrl->out_reserve[d * kp.nsub + k].v, 1ull);
     pidx = __shfl_sync(kFull, pidx, 0);
-    const uint32_t slot = (uint32_t)(pidx & (cp - 1));
+    const uint32_t slot = sub_slot(kp, k, pidx);
     uint64_t t_begin = 0;
     for (;;) {   // wait for the receiver to free the slot; keep consuming inbound meanwhile
         int st = 0;
@@ -422,22 +429,22 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
     const RankDev &R = s.R;
     if (R.n_ranks <= 1) return false;
     const int lane = threadIdx.x & 31;
-    const uint32_t cp = (uint32_t)kp.cp;
-    const int p = R.n_ranks;
-    const int start = (w + (int)(s.c_idle & 7)) % p;
-    for (int k = 0; k < p; ++k) {
-        const int sr = (start + k) % p;
+    const uint32_t cps = (uint32_t)kp.cps;
+    const int p = R.n_ranks, nc = p * kp.nsub;
+    const int start = (w + (int)(s.c_idle & 7)) % nc;
+    for (int kk = 0; kk < nc; ++kk) {
+        const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
         if (sr == R.rank) continue;
-        unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[sr].v;
+        unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
         uint64_t cc = 0;
         if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
         cc = __shfl_sync(kFull, cc, 0);
         bool ready = false;
         uint32_t cnt = 0;
-        if (lane < kClaim && (uint32_t)lane < cp) {
+        if (lane < kClaim && (uint32_t)lane < cps) {
             // relaxed poll: an acquire load also invalidates L1 (CCTL.IVALL), which
             // every idle warp would otherwise do on every poll of every channel
-            const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+            const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);
             ready = hi32(h) == lo32(cc + lane + 1);
             cnt = lo32(h);
         }
@@ -449,12 +456,12 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
         if (!__shfl_sync(kFull, won, 0)) continue;
         // acquire each claimed header (synchronises with its sender's st.release),
         // then the warp barrier orders every lane's payload reads after them
-        if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);
+        if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);
         __syncwarp();
         uint32_t total = 0;
         for (int q = 0; q < r; ++q) {
             const uint32_t cq = __shfl_sync(kFull, cnt, q);
-            const uint32_t slot = (uint32_t)((cc + q) & (cp - 1));
+            const uint32_t slot = sub_slot(kp, sk, cc + q);
             const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
             for (uint32_t base = 0; base < cq; base += 32 * kInU) {
                 bool pred[kInU];
@@ -512,7 +519,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
             // handed back to the sender and before R counts the messages
             fence_peer(kp.sys);
             for (int q = 0; q < r; ++q)
-                st_relaxed_peer(kp.sys, &R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);   // slots free for the sender
+                st_relaxed_peer(kp.sys, &R.peer_free[sr][sub_slot(kp, sk, cc + q)], cc + q + cps);   // slots free for the sender
             atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)total);
         }
         __syncwarp();
@@ -530,22 +537,22 @@ template <int APP>
 __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint32_t cp = (uint32_t)kp.cp;
+    const uint32_t cps = (uint32_t)kp.cps;
     if (w == 0) {
-        const int p = R.n_ranks;
-        const int start = (cta + (int)s.c_idle) % p;
+        const int nc = R.n_ranks * kp.nsub;
+        const int start = (cta + (int)s.c_idle) % nc;
         int got = 0;
-        for (int k = 0; k < p && !got; ++k) {
-            const int sr = (start + k) % p;
+        for (int kk = 0; kk < nc && !got; ++kk) {
+            const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
             if (sr == R.rank) continue;
-            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[sr].v;
+            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
             uint64_t cc = 0;
             if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
             cc = __shfl_sync(kFull, cc, 0);
             bool ready = false;
             uint32_t cnt = 0;
-            if (lane < kClaim && (uint32_t)lane < cp) {
-                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // relaxed poll
+            if (lane < kClaim && (uint32_t)lane < cps) {
+                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
                 ready = hi32(h) == lo32(cc + lane + 1);
                 cnt = lo32(h);
             }
@@ -555,7 +562,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
             int won = 0;
             if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
             if (!__shfl_sync(kFull, won, 0)) continue;
-            if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][(cc + lane) & (cp - 1)]);   // sync with each sender's release
+            if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // sync with each sender's release
             uint32_t incl = lane < r ? cnt : 0u;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
@@ -563,14 +570,14 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                 if (lane >= d) incl += y;
             }
             if (lane < r) s.in_off[lane + 1] = incl;
-            if (lane == 0) { s.in_off[0] = 0; s.in_src = sr; s.in_cc = cc; s.in_r = r; }
+            if (lane == 0) { s.in_off[0] = 0; s.in_src = ch; s.in_cc = cc; s.in_r = r; }
             got = 1;
         }
         if (lane == 0) s.in_got = got;
     }
     __syncthreads();      // also orders warp 0's acquires before every thread's payload reads
     if (!s.in_got) return false;
-    const int sr = s.in_src, r = s.in_r;
+    const int ch = s.in_src, sr = ch / kp.nsub, sk = ch % kp.nsub, r = s.in_r;
     const uint64_t cc = s.in_cc;
     const uint32_t M = s.in_off[r];
     uint32_t wn = s.wn[w];
@@ -585,7 +592,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
             ul[j] = 0;
             if (m < M) {
                 while (q + 1 < r && s.in_off[q + 1] <= m) ++q;   // packet holding message m
-                const uint32_t slot = (uint32_t)((cc + q) & (cp - 1));
+                const uint32_t slot = sub_slot(kp, sk, cc + q);
                 const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
                 const uint32_t i = m - s.in_off[q];
                 if constexpr (APP == kApBfs) {
@@ -617,7 +624,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
         // ordered before the slots go back to the sender and before R counts them
         fence_peer(kp.sys);
         for (int q = 0; q < r; ++q)
-            st_relaxed_peer(kp.sys, &R.peer_free[sr][(cc + q) & (cp - 1)], cc + q + cp);
+            st_relaxed_peer(kp.sys, &R.peer_free[sr][sub_slot(kp, sk, cc + q)], cc + q + cps);
         atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)M);
         s.c_batches++;
     }
@@ -949,6 +956,107 @@ __device__ void expand_warp_pipe(Smem &s, BatchBuf &bb, const KParams &kp, int c
     }
 }
 
+// ---------------------------------------------------------------------------
+// BFS expansion, three-stage software pipeline (pipeline = 3): while chunk i
+// is relaxed (compare, red/atomicMin, append), the probes of chunk i+1 and the
+// column loads of chunk i+2 are already in flight, so a warp keeps two memory
+// round trips outstanding instead of waiting on col -> probe per chunk.  No hub
+// cache (the caller falls back to expand_warp when it is on).
+// ---------------------------------------------------------------------------
+template <bool MULTI>
+__device__ __forceinline__ void probe_issue(const KParams &kp, const RankDev &R, const PipeStage &st,
+                                            uint32_t (&cur)[kPU]) {
+#pragma unroll
+    for (int k = 0; k < kPU; ++k)
+        cur[k] = st.u[k] < 0 ? 0u : (kp.filter ? ldg_u8(R.filt + st.u[k]) : ldg_u32(R.depth + st.u[k]));
+}
+
+template <int APP, bool MULTI>
+__device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta, PipeStage &st,
+                                             const uint32_t (&cur)[kPU], uint32_t &wn) {
+    const RankDev &R = s.R;
+    const int w = threadIdx.x >> 5;
+    const int64_t vb = R.v_begin, ve = R.v_end;
+    const bool fl = kp.filter;
+    bool imp[kPU];
+#pragma unroll
+    for (int k = 0; k < kPU; ++k) {
+        const uint32_t nd = st.nd[k], ndw = dw_make(nd);
+        const bool maybe = st.u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k]);
+        imp[k] = false;
+        if (maybe) {
+            if (kp.relax_red) {
+                red_min_u32(R.depth + st.u[k], ndw);
+                imp[k] = true;
+            } else {
+                imp[k] = atom_min_u32(R.depth + st.u[k], ndw) > ndw;
+            }
+            if (fl && imp[k]) stg_u8(R.filt + st.u[k], filt_of(nd));
+        }
+    }
+    if constexpr (!MULTI) {
+        uint32_t msk = 0, item[kPU];
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) {
+            msk |= (imp[k] ? 1u : 0u) << k;
+            item[k] = (uint32_t)(st.u[k] - vb);
+        }
+        warp_append_mask<kPU>(s, w, wn, msk, item, kp.relax_red);
+    } else {
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) {
+            const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
+            if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
+            warp_append_local(s, w, wn, loc, (uint32_t)(st.u[k] - vb));
+            const bool rem = imp[k] && !loc;
+            const int d = rem ? owner_of(R, st.u[k]) : 0;
+            warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
+                                    (uint64_t)st.nd[k], wn);
+        }
+    }
+}
+
+template <int APP, bool MULTI>
+__device__ void expand_warp_pipe3(Smem &s, BatchBuf &bb, const KParams &kp, int cta, int B, int64_t E, uint32_t &wn) {
+    const int lane = threadIdx.x & 31;
+    const RankDev &R = s.R;
+    const int32_t *const col = R.col;
+    const uint64_t pol = policy_evict_first();
+    const uint32_t nchm = (uint32_t)((E + kChunk - 1) / kChunk);
+    const uint32_t nch = (uint32_t)((E + kPChunk - 1) / kPChunk);
+    auto claim = [&]() {
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
+        return __shfl_sync(kFull, c, 0);
+    };
+    PipeStage a, b, c;
+    uint32_t ca = claim();
+    if (ca >= nch) return;
+    pipe_load(bb, B, E, nchm, ca, a, col, pol);
+    uint32_t cb = claim();
+    const bool hb = cb < nch;
+    if (hb) pipe_load(bb, B, E, nchm, cb, b, col, pol);
+    uint32_t cur_a[kPU], cur_b[kPU];
+    probe_issue<MULTI>(kp, R, a, cur_a);
+    bool have_b = hb;
+    for (;;) {
+        bool have_c = false;
+        if (have_b) {
+            const uint32_t cc = claim();
+            have_c = cc < nch;
+            if (have_c) pipe_load(bb, B, E, nchm, cc, c, col, pol);   // columns of chunk i+2
+            probe_issue<MULTI>(kp, R, b, cur_b);                     // probes of chunk i+1
+        }
+        relax_finish<APP, MULTI>(s, kp, cta, a, cur_a, wn);          // chunk i
+        if (!have_b) break;
+        a = b;
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) cur_a[k] = cur_b[k];
+        b = c;
+        have_b = have_c;
+    }
+}
+
 // Load per-vertex info of the batch s.v[0..B) and expand it.
 template <int APP, bool MULTI>
 __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
@@ -1033,6 +1141,11 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         const int w = tid >> 5;
         uint32_t wn = s.wn[w];
         // pipelined expansion pays off on low-degree (latency-bound, road-like) batches
+#ifdef ATOS_PIPE3   // experimental: raises register pressure (stack spills) of the default paths
+        if (APP == kApBfs && kp.pipe == 3 && kp.hc_per_rank == 0)
+            expand_warp_pipe3<APP, MULTI>(s, bb, kp, cta, B, E, wn);
+        else
+#endif
         if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
             expand_warp_pipe<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         else expand_warp<APP, MULTI>(s, bb, kp, cta, B, E, wn);
