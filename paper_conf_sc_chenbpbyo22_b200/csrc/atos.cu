@@ -384,6 +384,27 @@ __global__ void permute_rows_kernel(const int64_t *rp_old, const int32_t *col_ol
     }
 }
 
+// Streamed variant for a host column array: old rows [l0, l1) restricted to the
+// staged column range [c0, c1) (rank-relative offsets), one warp per old row;
+// column ids are range-checked here (they are never checked elsewhere on this path).
+__global__ void permute_chunk_kernel(const int64_t *rp_old, const int32_t *stage, int64_t c0, int64_t c1,
+                                     int64_t l0, int64_t l1, const int32_t *perm, int64_t v0,
+                                     const int64_t *rp_new, int32_t *col_new, int64_t n, unsigned long long *bad) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t l = l0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); l < l1; l += nw) {
+        const int64_t b = rp_old[l], e = rp_old[l + 1];
+        const int64_t lo = b > c0 ? b : c0, hi = e < c1 ? e : c1;
+        if (lo >= hi) continue;
+        const int64_t o = rp_new[perm[v0 + l] - v0] + (lo - b);
+        for (int64_t k = lane; k < hi - lo; k += 32) {
+            int32_t x = stage[lo - c0 + k];
+            if (x < 0 || (int64_t)x >= n) { atomicOr(bad, 2ull); x = 0; }
+            col_new[o + k] = perm[x];
+        }
+    }
+}
+
 static bool is_device_ptr(const void *p) {
     if (!p) return false;
     cudaPointerAttributes a;
@@ -539,6 +560,96 @@ static atos_status relabel_rows(atos_graph *g, LocalRank &me) {
     return ATOS_OK;
 }
 
+// Relabeled rows of rank `me` straight from a HOST column array: the columns are
+// streamed in chunks through two device staging buffers on a second stream, and
+// each chunk is permuted into place while the next one is copied, so the H2D
+// transfer (the dominant cost of an end-to-end load) overlaps the permutation
+// instead of preceding it.  me.row_ptr must be copied, rebased and validated.
+static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int64_t *rp_host, const int32_t *col_host,
+                                         unsigned long long *d_bad) {
+    cudaStream_t st = g->stream;
+    const int r = me.rank;
+    const int64_t v0 = g->part[r], nr = me.L.n_r, m = me.m_r, base = rp_host[v0];
+    DevFrees fr;
+    int64_t *deg = nullptr, *rp_new = nullptr;
+    int32_t *col_new = nullptr;
+    CU(cudaMalloc(&deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
+    CU(cudaMalloc(&rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
+    CU(cudaMalloc(&col_new, (size_t)std::max<int64_t>(m, 1) * 4)); fr.p.push_back(col_new);
+    new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
+    size_t tb = 0;
+    CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
+    void *tmp = nullptr;
+    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    fr.p.push_back(tmp);
+    CU(cub::DeviceScan::ExclusiveSum(tmp, tb, deg, rp_new, (int64_t)(nr + 1), st));
+    int64_t ch = (int64_t)1 << 26;                  // 256 MB per stage
+    if (const char *e = std::getenv("ATOS_LOAD_CHUNK")) ch = std::max<int64_t>(1, std::atoll(e));   // tests: many chunks
+    const int64_t CH = std::min<int64_t>(std::max<int64_t>(m, 1), ch);
+    int32_t *stage[2] = {nullptr, nullptr};
+    for (int k = 0; k < 2; ++k) { CU(cudaMalloc(&stage[k], (size_t)CH * 4)); fr.p.push_back(stage[k]); }
+    cudaStream_t cs = nullptr;
+    CU(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    cudaEvent_t ev_in[2], ev_out[2], ev_ready;
+    for (int k = 0; k < 2; ++k) {
+        CU(cudaEventCreateWithFlags(&ev_in[k], cudaEventDisableTiming));
+        CU(cudaEventCreateWithFlags(&ev_out[k], cudaEventDisableTiming));
+    }
+    CU(cudaEventCreateWithFlags(&ev_ready, cudaEventDisableTiming));
+    CU(cudaEventRecord(ev_ready, st));           // rp_new and the row offsets are ready
+    CU(cudaStreamWaitEvent(cs, ev_ready, 0));
+    atos_status status = ATOS_OK;
+    const bool trace = std::getenv("ATOS_LOAD_TRACE") != nullptr;
+    std::vector<cudaEvent_t> tev;
+    auto tmark = [&](cudaStream_t s_) {
+        if (!trace) return;
+        cudaEvent_t e_;
+        cudaEventCreate(&e_);
+        cudaEventRecord(e_, s_);
+        tev.push_back(e_);
+    };
+    for (int64_t c0 = 0, k = 0; c0 < m && status == ATOS_OK; c0 += CH, ++k) {
+        const int64_t c1 = std::min(m, c0 + CH);
+        const int b = (int)(k & 1);
+        // rows overlapping [c0, c1): first row ending after c0 .. first row starting at/after c1
+        const int64_t *rp = rp_host + v0;
+        const int64_t l0 = (int64_t)(std::upper_bound(rp, rp + nr + 1, base + c0) - rp) - 1;
+        const int64_t l1 = (int64_t)(std::lower_bound(rp, rp + nr + 1, base + c1) - rp);
+        if (k >= 2 && cudaStreamWaitEvent(cs, ev_out[b], 0) != cudaSuccess) status = fail(ATOS_ERR_CUDA, "stream wait");
+        tmark(cs);
+        if (cudaMemcpyAsync(stage[b], col_host + base + c0, (size_t)(c1 - c0) * 4, cudaMemcpyHostToDevice, cs) != cudaSuccess)
+            status = fail(ATOS_ERR_CUDA, "cudaMemcpyAsync of a column chunk failed");
+        tmark(cs);
+        cudaEventRecord(ev_in[b], cs);
+        cudaStreamWaitEvent(st, ev_in[b], 0);
+        tmark(st);
+        permute_chunk_kernel<<<2048, 256, 0, st>>>(me.row_ptr, stage[b], c0, c1, std::max<int64_t>(l0, 0),
+                                                  std::min(l1, nr), g->d_perm, v0, rp_new, col_new, g->n, d_bad);
+        tmark(st);
+        cudaEventRecord(ev_out[b], st);
+    }
+    const cudaError_t e = cudaStreamSynchronize(st);
+    cudaStreamSynchronize(cs);
+    for (size_t i = 0; i + 3 < tev.size(); i += 4) {
+        float a = 0, b2 = 0;
+        cudaEventElapsedTime(&a, tev[i], tev[i + 1]);
+        cudaEventElapsedTime(&b2, tev[i + 2], tev[i + 3]);
+        fprintf(stderr, "[atos load]   chunk %zu: copy %.2f ms, permute %.2f ms\n", i / 4, a, b2);
+    }
+    for (cudaEvent_t x : tev) cudaEventDestroy(x);
+    for (int k = 0; k < 2; ++k) { cudaEventDestroy(ev_in[k]); cudaEventDestroy(ev_out[k]); }
+    cudaEventDestroy(ev_ready);
+    cudaStreamDestroy(cs);
+    if (status != ATOS_OK) return status;
+    if (e != cudaSuccess) return fail(ATOS_ERR_CUDA, "streamed relabel: %s", cudaGetErrorString(e));
+    cudaFree(me.row_ptr);
+    me.row_ptr = rp_new;
+    me.col = col_new;
+    fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)rp_new), fr.p.end());
+    fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)col_new), fr.p.end());
+    return ATOS_OK;
+}
+
 extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *col, int64_t n, int64_t nnz,
                                        const int64_t *part, const atos_config *cfg_in, atos_graph **out) {
     if (!out) return fail(ATOS_ERR_INVALID_ARG, "out is NULL");
@@ -653,16 +764,27 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         CU(cudaMalloc(&me.arena, me.L.total));
         CU(cudaMemsetAsync(me.arena, 0, me.L.total, g->stream));
         tr.mark(g->stream, "arena");
+        // host CSR + relabeling: stream the columns through the permutation (no
+        // full-size device copy of the unpermuted columns)
+        const bool streamed = g->d_perm && me.m_r > 0 && !rp_dev && !is_device_ptr(col);
         CU(cudaMalloc(&me.row_ptr, (size_t)(nr + 1) * 8));
-        CU(cudaMalloc(&me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
+        if (!streamed) CU(cudaMalloc(&me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
         CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
-        if (me.m_r > 0)
+        if (me.m_r > 0 && !streamed)
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
         tr.mark(g->stream, "copy csr");
         rebase_rows_kernel<<<256, 256, 0, g->stream>>>(me.row_ptr, nr + 1, rb[r]);
-        check_rows_kernel<<<1024, 256, 0, g->stream>>>(me.row_ptr, nr, me.m_r, me.col, n, d_bad);
+        check_rows_kernel<<<1024, 256, 0, g->stream>>>(me.row_ptr, nr, streamed ? 0 : me.m_r, me.col, n, d_bad);
         tr.mark(g->stream, "check rows");
-        if (g->d_perm) {   // rows must be valid before they are permuted
+        if (streamed) {
+            unsigned long long bad0 = 0;
+            CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
+            CU(cudaStreamSynchronize(g->stream));
+            if (bad0) { cudaFree(d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone"); }
+            atos_status rs = relabel_rows_streamed(g, me, row_ptr, col, d_bad);
+            if (rs != ATOS_OK) { cudaFree(d_bad); return rs; }
+            tr.mark(g->stream, "relabel rows (streamed)");
+        } else if (g->d_perm) {   // rows must be valid before they are permuted
             unsigned long long bad0 = 0;
             CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
             CU(cudaStreamSynchronize(g->stream));
@@ -755,7 +877,8 @@ static KParams make_params(atos_graph *g) {
     // probe filter: explicit, or automatically when the depth words do not fit the
     // L2 persisting carve-out (RMAT-26: 268 MB of words, 67 MB of filter)
     kp.filter = g->cfg.probe_filter == 1 ||
-                (g->cfg.probe_filter == 2 && (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20));
+                (g->cfg.probe_filter == 2 && (g->skewed ||
+                                              (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20)));
     kp.hc_per_rank = g->hc_per_rank;
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;

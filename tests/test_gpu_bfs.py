@@ -278,3 +278,19 @@ def test_discrete_iterations_equal_levels_on_a_path():
         assert np.array_equal(d2, np.arange(n)[::-1]) and st2["iterations"] == n
     with pytest.raises(atos.AtosError):
         atos.Graph(rp, col, discrete=1, virtual_ranks=2)
+
+
+@pytest.mark.parametrize("chunk", ["7", "1000", "100003"])
+def test_streamed_relabel_load_from_host(chunk, monkeypatch):
+    """Host CSR + relabeling streams the columns through the permutation in chunks
+    (graph_load); chunk boundaries inside rows must not change anything."""
+    monkeypatch.setenv("ATOS_LOAD_CHUNK", chunk)
+    g = inputs.rmat(14, 16, 8, symmetric=True)
+    rp, col = g.numpy()
+    for s in inputs.bfs_sources(g, 2, seed=4):
+        run_and_check(rp, col, s, relabel=1)
+    bad = col.copy()
+    bad[len(bad) // 2] = g.n + 5                        # out-of-range column id inside a late chunk
+    with pytest.raises(atos.AtosError) as e:
+        atos.Graph(rp, bad, relabel=1)
+    assert e.value.status == 1
