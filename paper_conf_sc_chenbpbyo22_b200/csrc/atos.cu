@@ -882,7 +882,8 @@ static KParams make_params(atos_graph *g) {
     kp.hc_per_rank = g->hc_per_rank;
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
-    kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
+    kp.sys = g->multiproc ? 1 : 0;
+    kp.early = std::getenv("ATOS_NO_EARLY") ? 0 : 1;   // experiment switch   // virtual ranks share this device: .gpu scope suffices
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;
