@@ -31,6 +31,10 @@
 
 namespace atos {
 
+#ifndef ATOS_MINB
+#define ATOS_MINB (1024 / ATOS_THREADS)
+#endif
+constexpr int kMinBlocks = ATOS_MINB;   // resident CTAs per SM the register budget is sized for
 constexpr int kApBfs = 0;
 constexpr int kApPr = 1;
 #ifndef ATOS_KU
@@ -42,8 +46,7 @@ constexpr int kChunk = 32 * kU;      // edges per warp chunk
 #define ATOS_WOUT 256
 #endif
 constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
-constexpr int kChunkMap = 1024;
-constexpr int kClaimMax = 8;         // packets one warp claims from a sub-channel at once      // chunks whose first vertex is precomputed per batch
+constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr int kHubMax = 65536;       // max hub-cache entries per CTA (32 KB of nibbles; 2 CTAs/SM still fit)
 
@@ -99,10 +102,9 @@ struct Smem {
     uint64_t wave[kMaxRanks][5];   // coordinator double wave
     int32_t wave_valid;
     // CTA-cooperative inbound claim (cta_inbound)
-    struct InClaim { int32_t ch, r; uint64_t cc; uint32_t off[kClaimMax + 1]; };
-    InClaim in_claim[kWarps];      // claims of this iteration (at most one per warp)
-    int32_t in_n;
-    uint64_t in_cache[kMaxRanks * kMaxSub];   // last known cursor of every inbound sub-channel
+    int32_t in_got, in_src, in_r;
+    uint64_t in_cc;
+    uint32_t in_off[33];
     unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
 #ifdef ATOS_PROF
     unsigned long long prof[10];
@@ -530,50 +532,40 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
     return false;
 }
 
-// Whole CTA (the worker loop's receive step).  Every warp polls its own share
-// of the inbound sub-channels IN PARALLEL (lane-parallel header probes at the
-// cached cursor, so one round trip) and claims the ready prefix (up to
-// kClaimMax packets) of at most one with one CAS; then ALL 512 threads apply the
-// claimed messages -- a claim is expanded like a pop batch.  Sequential polling
-// of p x nsub channels by one warp kept the other 15 at the loop barrier.
-// Returns whether anything was claimed (CTA-uniform).
+// Whole CTA (the worker loop's receive step): warp 0 claims the ready prefix (up
+// to kClaim packets) of one inbound channel with one CAS, then ALL 512 threads
+// apply its messages -- a claimed set is expanded like a pop batch, instead of one
+// warp applying it while the other 15 wait at the loop's barrier.  Returns
+// whether anything was claimed (CTA-uniform).
 template <int APP>
 __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const uint32_t cps = (uint32_t)kp.cps;
-    const int nc = R.n_ranks * kp.nsub;
-    if (tid == 0) s.in_n = 0;
-    __syncthreads();
-    {
-        const int rot = (cta + (int)s.c_idle) % nc;
-        for (int ci = w; ci < nc; ci += kWarps) {
-            const int ch = (ci + rot) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
+    if (w == 0) {
+        const int nc = R.n_ranks * kp.nsub;
+        const int start = (cta + (int)s.c_idle) % nc;
+        int got = 0;
+        for (int kk = 0; kk < nc && !got; ++kk) {
+            const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
             if (sr == R.rank) continue;
-            const uint64_t cc = s.in_cache[ch];
-            bool ready = false, ahead = false;
+            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+            uint64_t cc = 0;
+            if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+            cc = __shfl_sync(kFull, cc, 0);
+            bool ready = false;
             uint32_t cnt = 0;
-            if (lane < kClaimMax && (uint32_t)lane < cps) {
+            if (lane < kClaim && (uint32_t)lane < cps) {
                 const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
                 ready = hi32(h) == lo32(cc + lane + 1);
-                ahead = (int32_t)(hi32(h) - lo32(cc + lane + 1)) > 0;   // slot reused by a later lap: cache is stale
                 cnt = lo32(h);
-            }
-            if (__shfl_sync(kFull, ahead, 0)) {
-                if (lane == 0) s.in_cache[ch] = ld_relaxed_gpu(&R.ctrl->in_cursor[ch].v);
-                continue;
             }
             const uint32_t nready = __ballot_sync(kFull, ready);
             const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
             if (r == 0) continue;
-            unsigned long long o = 0;
-            if (lane == 0) o = atomicCAS((unsigned long long *)&R.ctrl->in_cursor[ch].v, (unsigned long long)cc,
-                                         (unsigned long long)(cc + r));
-            o = __shfl_sync(kFull, o, 0);
-            if (o != cc) {                     // another worker moved the cursor: refresh the cache
-                if (lane == 0 && o > s.in_cache[ch]) s.in_cache[ch] = o;
-                continue;
-            }
+            int won = 0;
+            if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+            if (!__shfl_sync(kFull, won, 0)) continue;
             if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // sync with each sender's release
             uint32_t incl = lane < r ? cnt : 0u;
 #pragma unroll
@@ -581,79 +573,63 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                 const uint32_t y = __shfl_up_sync(kFull, incl, d);
                 if (lane >= d) incl += y;
             }
-            int slot_i = 0;
-            if (lane == 0) {
-                slot_i = atomicAdd(&s.in_n, 1);
-                s.in_cache[ch] = cc + r;
-            }
-            slot_i = __shfl_sync(kFull, slot_i, 0);
-            Smem::InClaim &c = s.in_claim[slot_i];
-            if (lane < r) c.off[lane + 1] = incl;
-            if (lane == 0) { c.off[0] = 0; c.ch = ch; c.cc = cc; c.r = r; }
-            break;                             // one claim per warp per iteration
+            if (lane < r) s.in_off[lane + 1] = incl;
+            if (lane == 0) { s.in_off[0] = 0; s.in_src = ch; s.in_cc = cc; s.in_r = r; }
+            got = 1;
         }
+        if (lane == 0) s.in_got = got;
     }
-    __syncthreads();      // also orders the claimers' acquires before every thread's payload reads
-    const int nclaims = s.in_n;
-    if (nclaims == 0) return false;
+    __syncthreads();      // also orders warp 0's acquires before every thread's payload reads
+    if (!s.in_got) return false;
+    const int ch = s.in_src, sr = ch / kp.nsub, sk = ch % kp.nsub, r = s.in_r;
+    const uint64_t cc = s.in_cc;
+    const uint32_t M = s.in_off[r];
     uint32_t wn = s.wn[w];
-    for (int ci = 0; ci < nclaims; ++ci) {
-        const Smem::InClaim &c = s.in_claim[ci];
-        const int ch = c.ch, sr = ch / kp.nsub, sk = ch % kp.nsub, r = c.r;
-        const uint64_t cc = c.cc;
-        const uint32_t M = c.off[r];
-        for (uint32_t base = 0; base < M; base += kThreads * kInU) {
-            bool pred[kInU];
-            uint32_t ul[kInU];
-            int q = 0;
+    for (uint32_t base = 0; base < M; base += kThreads * kInU) {
+        bool pred[kInU];
+        uint32_t ul[kInU];
+        int q = 0;
 #pragma unroll
-            for (int j = 0; j < kInU; ++j) {
-                const uint32_t m = base + j * kThreads + tid;
-                pred[j] = false;
-                ul[j] = 0;
-                if (m < M) {
-                    while (q + 1 < r && c.off[q + 1] <= m) ++q;   // packet holding message m
-                    const uint32_t slot = sub_slot(kp, sk, cc + q);
-                    const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
-                    const uint32_t i = m - c.off[q];
-                    if constexpr (APP == kApBfs) {
-                        const uint64_t msg = ld_cg_u64((const uint64_t *)pay + i);
-                        ul[j] = lo32(msg);
-                        const uint32_t ndw = dw_make(hi32(msg));
-                        pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
-                        if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(msg)));
-                    } else {
-                        const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
-                        ul[j] = msg.x;
-                        const double dlt = __longlong_as_double((long long)(((uint64_t)msg.w << 32) | msg.z));
-                        const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
-                        pred[j] = old < kp.eps && old + dlt >= kp.eps;
-                    }
+        for (int j = 0; j < kInU; ++j) {
+            const uint32_t m = base + j * kThreads + tid;
+            pred[j] = false;
+            ul[j] = 0;
+            if (m < M) {
+                while (q + 1 < r && s.in_off[q + 1] <= m) ++q;   // packet holding message m
+                const uint32_t slot = sub_slot(kp, sk, cc + q);
+                const unsigned char *pay = R.in_payload[sr] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+                const uint32_t i = m - s.in_off[q];
+                if constexpr (APP == kApBfs) {
+                    const uint64_t msg = ld_cg_u64((const uint64_t *)pay + i);
+                    ul[j] = lo32(msg);
+                    const uint32_t ndw = dw_make(hi32(msg));
+                    pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
+                    if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(msg)));
+                } else {
+                    const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
+                    ul[j] = msg.x;
+                    const double dlt = __longlong_as_double((long long)(((uint64_t)msg.w << 32) | msg.z));
+                    const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
+                    pred[j] = old < kp.eps && old + dlt >= kp.eps;
                 }
             }
+        }
 #pragma unroll
-            for (int j = 0; j < kInU; ++j) {
-                if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
-                warp_append_local(s, w, wn, pred[j], ul[j]);
-            }
+        for (int j = 0; j < kInU; ++j) {
+            if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, false);
+            warp_append_local(s, w, wn, pred[j], ul[j]);
         }
     }
     warp_flush_local(s, w, wn, false);        // T counts the new local work before R
     if (lane == 0) s.wn[w] = wn;
     __syncthreads();
     if (tid == 0) {
-        // one fence per iteration: payload reads and their effects are ordered
-        // before the slots go back to the senders and before R counts them
+        // one system-scope fence per claim: payload reads and their effects are
+        // ordered before the slots go back to the sender and before R counts them
         fence_peer(kp.sys);
-        uint64_t tot = 0;
-        for (int ci = 0; ci < nclaims; ++ci) {
-            const Smem::InClaim &c = s.in_claim[ci];
-            const int sr = c.ch / kp.nsub, sk = c.ch % kp.nsub;
-            for (int q = 0; q < c.r; ++q)
-                st_relaxed_peer(kp.sys, &R.peer_free[sr][sub_slot(kp, sk, c.cc + q)], c.cc + q + cps);
-            tot += c.off[c.r];
-        }
-        atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)tot);
+        for (int q = 0; q < r; ++q)
+            st_relaxed_peer(kp.sys, &R.peer_free[sr][sub_slot(kp, sk, cc + q)], cc + q + cps);
+        atomicAdd((unsigned long long *)&R.ctrl->recvd.v, (unsigned long long)M);
         s.c_batches++;
     }
     return true;
@@ -1401,14 +1377,10 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = 0;
         s.c_busy = s.c_batches = 0;
         s.limit = kp.discrete ? ld_relaxed_gpu(&s.R.ctrl->limit.v) : 0;
-        s.in_n = 0;
 #ifdef ATOS_PROF
         for (int k = 0; k < 10; ++k) s.prof[k] = 0;
 #endif
     }
-    if (MULTI)   // cursor cache: start from the current cursors
-        for (int ch = tid; ch < kMaxRanks * kMaxSub; ch += kThreads)
-            s.in_cache[ch] = ld_relaxed_gpu(&kp.ranks[lr].ctrl->in_cursor[ch].v);
     if (tid < kWarps) {
         s.wn[tid] = 0;
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
@@ -1531,7 +1503,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
 
 // The persistent worker (one cooperative launch per solve).
 template <int APP, bool MULTI>
-__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KParams kp) {
+__global__ void __launch_bounds__(kThreads, kMinBlocks) worker_kernel(KParams kp) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     worker_body<APP, MULTI>(*reinterpret_cast<Smem *>(smem_raw), kp);
 }
@@ -1540,7 +1512,7 @@ __global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_kernel(KPara
 // a CUDA-graph while-node; the per-solve parameters live in device memory so the
 // instantiated graph never changes.
 template <int APP>
-__global__ void __launch_bounds__(kThreads, 1024 / kThreads) worker_discrete_kernel(const KParams *kpp) {
+__global__ void __launch_bounds__(kThreads, kMinBlocks) worker_discrete_kernel(const KParams *kpp) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ KParams kps;
     if (threadIdx.x == 0) kps = *kpp;

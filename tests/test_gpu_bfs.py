@@ -294,3 +294,60 @@ def test_streamed_relabel_load_from_host(chunk, monkeypatch):
     with pytest.raises(atos.AtosError) as e:
         atos.Graph(rp, bad, relabel=1)
     assert e.value.status == 1
+
+
+def bfs_properties_hold(rp_dev, col_dev, depth_dev, src):
+    """Properties that fix BFS depths on a symmetric graph at any size (checked on
+    the GPU with plain torch ops): depth(src) = 0; |d(u) - d(v)| <= 1 on every edge
+    between reached vertices; no edge from a reached to an unreached vertex; every
+    reached v != src has a neighbour at depth d(v) - 1."""
+    n = rp_dev.numel() - 1
+    deg = rp_dev[1:] - rp_dev[:-1]
+    d = depth_dev.to(torch.int64)
+    assert int(d[src]) == 0
+    ok_all = True
+    # process the edge list in slices to bound memory
+    row = torch.repeat_interleave(torch.arange(n, device=d.device), deg)
+    has_parent = torch.zeros(n, dtype=torch.bool, device=d.device)
+    step = 1 << 28
+    for a in range(0, col_dev.numel(), step):
+        u = row[a:a + step]
+        v = col_dev[a:a + step].to(torch.int64)
+        du, dv = d[u], d[v]
+        ru, rv = du >= 0, dv >= 0
+        ok_all &= bool(((ru & rv) <= ((du - dv).abs() <= 1)).all())
+        ok_all &= bool((ru <= rv).all())
+        par = ru & rv & (du == dv - 1)
+        has_parent[v[par]] = True
+    reached = d >= 0
+    reached[src] = False
+    ok_all &= bool((reached <= has_parent).all())
+    return ok_all
+
+
+@pytest.mark.slow
+def test_rmat26_north_star_full_size():
+    """The north-star graph (RMAT-26 ef16 symmetric, 2.1 G CSR entries) in the bench's
+    launch configuration: bit-exact vs the oracle's serial BFS from one source, and
+    the BFS properties on the GPU from a second."""
+    g = inputs.make_config("rmat26", device="cuda")
+    srcs = inputs.bfs_sources(g, 2)
+    depth = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    with atos.Graph(g.row_ptr, g.col, g.n) as G:
+        G.bfs(srcs[1], depth_out=depth)
+        G.sync()
+        assert bfs_properties_hold(g.row_ptr, g.col, depth, srcs[1])
+        d0 = G.bfs(srcs[0])
+    rpn, coln = g.numpy()
+    assert np.array_equal(d0, oracle.bfs(rpn, coln, srcs[0]))
+
+
+@pytest.mark.slow
+def test_grid4900_config3_full_size():
+    """BASELINE configs[3] (road-like grid, 24 M vertices, ~11.8 K levels) at full size,
+    from the corner (the bench source) and the centre."""
+    g = inputs.make_config("grid4900", device="cuda")
+    rpn, coln = g.numpy()
+    with atos.Graph(g.row_ptr, g.col, g.n) as G:
+        for s in (0, g.n // 2 + 2450):
+            assert np.array_equal(G.bfs(s), oracle.bfs(rpn, coln, s))

@@ -157,3 +157,31 @@ def test_discrete_kernel_mode(graph):
         rp, col = csr_of(9, [(0, 1), (1, 2)])
     _, st = run_and_check(rp, col, discrete=1)
     assert st["iterations"] >= 1
+
+
+@pytest.mark.slow
+def test_rmat26_8ranks_config4_invariant_full_size():
+    """BASELINE configs[4] (PageRank RMAT-26 directed, 8 ranks -- virtual on one GPU,
+    as bench.py runs it) at full size, via properties that hold at any size: every
+    residual in [0, eps), and the push invariant
+        rank[v] + res[v] = (1 - alpha) + alpha * sum_{u -> v, outdeg(u) > 0} rank[u] / outdeg(u)
+    (rank grows only by residual that was pushed) to fp64 rounding.
+    With it, ||p_hat - p||_1 <= 2 * sum(res) / (1 - alpha) / sum(rank)."""
+    import torch
+    g = inputs.make_config("rmat26_pr", device="cuda")
+    n = g.n
+    r_out = torch.empty(n, dtype=torch.float64, device="cuda")
+    s_out = torch.empty(n, dtype=torch.float64, device="cuda")
+    with atos.Graph(g.row_ptr, g.col, n, relabel=0, virtual_ranks=8) as P:
+        P.pagerank(ALPHA, EPS, rank_out=r_out, residual_out=s_out)
+        P.sync()
+    assert bool((s_out >= 0).all()) and bool((s_out < EPS).all())
+    deg = (g.row_ptr[1:] - g.row_ptr[:-1]).to(torch.float64)
+    share = torch.where(deg > 0, r_out / deg.clamp(min=1), torch.zeros_like(r_out))
+    rhs = torch.full((n,), 1 - ALPHA, dtype=torch.float64, device="cuda")
+    row = torch.repeat_interleave(torch.arange(n, device="cuda"), g.row_ptr[1:] - g.row_ptr[:-1])
+    step = 1 << 28
+    for a in range(0, g.col.numel(), step):
+        rhs.index_add_(0, g.col[a:a + step].to(torch.int64), ALPHA * share[row[a:a + step]])
+    lhs = r_out + s_out
+    assert float((lhs - rhs).abs().max()) <= 1e-9 * max(1.0, float(lhs.abs().max()))
