@@ -871,6 +871,8 @@ static KParams make_params(atos_graph *g) {
     kp.keep = g->cfg.keep_items >= 0 ? g->cfg.keep_items
                                      : ((g->skewed || g->cfg.discrete || g->p > 1) ? 0 : kKeepAuto);
     kp.keep_always = g->cfg.keep_items >= 0 ? g->cfg.keep_mode : 1;
+    kp.keep_chain = 1 << 30;
+    if (const char *e = std::getenv("ATOS_KEEP_CHAIN")) kp.keep_chain = std::max(1, std::atoi(e));   // experiment
     kp.prefetch = g->cfg.prefetch;
     kp.relax_red = g->cfg.relax_red;
     kp.pipe = g->cfg.pipeline;
@@ -883,7 +885,9 @@ static KParams make_params(atos_graph *g) {
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
     kp.sys = g->multiproc ? 1 : 0;
-    kp.early = std::getenv("ATOS_NO_EARLY") ? 0 : 1;   // experiment switch   // virtual ranks share this device: .gpu scope suffices
+    // early next-batch reservation + per-warp enqueue: measured within noise
+    // (RMAT-24/26 BFS, RMAT-20 PR); off unless ATOS_EARLY is set (experiment)
+    kp.early = std::getenv("ATOS_EARLY") ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;

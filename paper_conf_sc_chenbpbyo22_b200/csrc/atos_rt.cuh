@@ -263,6 +263,7 @@ struct KParams {
     int32_t agg_on;
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
     int32_t keep_always;     // 1: keep whenever <= keep discovered; 0: only when the rank's T - F <= keep
+    int32_t keep_chain;      // max consecutive kept batches before the discoveries go to the ring
     int32_t prefetch;        // TMA bulk-prefetch each popped adjacency list into L2
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)

@@ -1420,6 +1420,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
 #endif
             if (B > 0) {
                 const int B0 = B;
+                int chain = 0;
                 while (B > 0) {                 // work-keeping chain
                     if (tid == 0) s.c_pops += B;
 #ifdef ATOS_PROF
@@ -1430,7 +1431,9 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
                     const long long pb2 = clock64();
                     if (tid == 0) s.prof[8] += (unsigned long long)(pb2 - pb1);
 #endif
-                    B = batch_end<APP, MULTI>(s, kp, cta, true);
+                    // a chain of kept batches is bounded (keep_chain): an unbounded
+                    // chain runs ahead of the wavefront and finds too-large depths
+                    B = batch_end<APP, MULTI>(s, kp, cta, ++chain < kp.keep_chain);
 #ifdef ATOS_PROF
                     if (tid == 0) s.prof[9] += (unsigned long long)(clock64() - pb2);
 #endif

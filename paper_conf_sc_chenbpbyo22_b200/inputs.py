@@ -258,6 +258,13 @@ def make_config(name: str, seed: int = 1, device="cpu", **override) -> CSR:
     cfg = dict(CONFIGS[name])
     cfg.update(override)
     if cfg["kind"] == "rmat":
-        return rmat(cfg["scale"], cfg["edgefactor"], seed, symmetric=cfg["symmetric"],
-                    permute=cfg["permute"], device=device)
-    return road_grid(cfg["W"], cfg["H"], seed, device=device)
+        g = rmat(cfg["scale"], cfg["edgefactor"], seed, symmetric=cfg["symmetric"],
+                 permute=cfg["permute"], device=device)
+    else:
+        g = road_grid(cfg["W"], cfg["H"], seed, device=device)
+    if str(device).startswith("cuda"):
+        # the generator's temporaries (edge lists, sort buffers: tens of GB at
+        # scale 26) stay in torch's cache otherwise, and libatos allocates with
+        # cudaMalloc outside that cache
+        torch.cuda.empty_cache()
+    return g
