@@ -55,7 +55,10 @@ def arm_config(args, g, srcs, world):
             "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
             "aggregation": bool(args.agg),
             "vertex_order": "degree-relabeled inside rank blocks (atos_config.relabel=auto); outputs in generator ids",
-            "l2": "no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9)}
+            "probe": "u8 depth-bound filter on skewed graphs (atos_config.probe_filter=auto)",
+            "l2": ("no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9))
+            if g.nnz * 4 + g.n * 8 > 126e6 else "CSR fits L2 (%.1f MB): a latency figure, not a bandwidth one"
+                                                % ((g.nnz * 4 + g.n * 8) / 1e6)}
 
 
 def log(*a):

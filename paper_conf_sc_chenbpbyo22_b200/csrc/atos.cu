@@ -240,6 +240,32 @@ struct atos_graph {
     cudaGraphExec_t dexec[2] = {nullptr, nullptr};
 };
 
+// Device memory of a handle comes from the device's default stream-ordered pool
+// with an unbounded release threshold, allocated and freed on the handle's
+// stream: a user loop that loads, solves and frees graphs (bench.py's e2e) reuses
+// physical memory instead of mapping and unmapping GBs through cudaMalloc /
+// cudaFree every time (measured 10-600 ms per call, varying).  The arena of a
+// multi-process handle stays on cudaMalloc: it is exported with cudaIpcGetMemHandle.
+static void pool_setup(int device) {
+    static bool done[64] = {false};
+    if (device < 0 || device >= 64 || done[device]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        done[device] = true;
+    } else {
+        cudaGetLastError();
+    }
+}
+template <typename T>
+static cudaError_t dmalloc(const atos_graph *g, T **p, size_t bytes) {
+    return cudaMallocAsync((void **)p, bytes, g->stream);
+}
+static void dfree(const atos_graph *g, void *p) {
+    if (p) cudaFreeAsync(p, g->stream);
+}
+
 // dynamic shared memory of the worker: Smem, plus the BFS hub cache (one nibble per entry)
 static size_t worker_smem(int app, int hc_entries) {
     return sizeof(Smem) + (app == kApBfs ? (size_t)hc_entries / 2 : 0);
@@ -430,15 +456,17 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     for (int s = 0; s < kMaxRanks; ++s)
         if (g->peer_opened[s]) cudaIpcCloseMemHandle(g->peer_base[s]);
     for (int lr = 0; lr < g->n_local; ++lr) {
-        cudaFree(g->loc[lr].arena);
-        cudaFree(g->loc[lr].row_ptr);
-        cudaFree(g->loc[lr].col);
+        if (g->multiproc) cudaFree(g->loc[lr].arena);
+        else dfree(g, g->loc[lr].arena);
+        dfree(g, g->loc[lr].row_ptr);
+        dfree(g, g->loc[lr].col);
     }
     cudaFree(g->d_ranks);
-    cudaFree(g->d_depth_full);
-    cudaFree(g->d_perm);
-    cudaFree(g->d_inv);
+    dfree(g, g->d_depth_full);
+    dfree(g, g->d_perm);
+    dfree(g, g->d_inv);
     cudaFree(g->d_accs);
+    if (g->stream) cudaStreamSynchronize(g->stream);
     for (int a = 0; a < 2; ++a) {
         if (g->dexec[a]) cudaGraphExecDestroy(g->dexec[a]);
         if (g->dgraph[a]) cudaGraphDestroy(g->dgraph[a]);
@@ -475,8 +503,10 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
 }
 
 struct DevFrees {   // scratch device buffers of graph_load, freed on every exit path
+    const atos_graph *g;
     std::vector<void *> p;
-    ~DevFrees() { for (void *x : p) cudaFree(x); }
+    explicit DevFrees(const atos_graph *g_) : g(g_) {}
+    ~DevFrees() { for (void *x : p) dfree(g, x); }
 };
 
 // Compute g->d_inv / g->d_perm (all rank blocks, identically on every process).
@@ -484,11 +514,11 @@ struct DevFrees {   // scratch device buffers of graph_load, freed on every exit
 static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool rp_dev) {
     const int64_t n = g->n;
     cudaStream_t st = g->stream;
-    DevFrees fr;
+    DevFrees fr(g);
     const int64_t *rpf = row_ptr;
     if (!rp_dev) {
         int64_t *t = nullptr;
-        CU(cudaMalloc(&t, (size_t)(n + 1) * 8));
+        CU(dmalloc(g, &t, (size_t)(n + 1) * 8));
         fr.p.push_back(t);
         CU(cudaMemcpyAsync(t, row_ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, st));
         rpf = t;
@@ -496,10 +526,10 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     uint32_t *k0 = nullptr, *k1 = nullptr;
     int32_t *v0 = nullptr;
     unsigned long long *d_max = nullptr;
-    CU(cudaMalloc(&k0, (size_t)n * 4)); fr.p.push_back(k0);
-    CU(cudaMalloc(&k1, (size_t)n * 4)); fr.p.push_back(k1);
-    CU(cudaMalloc(&v0, (size_t)n * 4)); fr.p.push_back(v0);
-    CU(cudaMalloc(&d_max, 8)); fr.p.push_back(d_max);
+    CU(dmalloc(g, &k0, (size_t)n * 4)); fr.p.push_back(k0);
+    CU(dmalloc(g, &k1, (size_t)n * 4)); fr.p.push_back(k1);
+    CU(dmalloc(g, &v0, (size_t)n * 4)); fr.p.push_back(v0);
+    CU(dmalloc(g, &d_max, 8)); fr.p.push_back(d_max);
     CU(cudaMemsetAsync(d_max, 0, 8, st));
     degree_keys_kernel<<<1024, 256, 0, st>>>(rpf, n, k0, v0, d_max);
     CU(cudaGetLastError());
@@ -510,14 +540,14 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     g->skewed = (double)mx >= 32.0 * std::max(1.0, mean);
     if (g->cfg.relabel == 0) return ATOS_OK;                           // degree statistics only
     if (g->cfg.relabel == 2 && !g->skewed) return ATOS_OK;              // not skewed: keep the given order
-    CU(cudaMalloc(&g->d_inv, (size_t)n * 4));
-    CU(cudaMalloc(&g->d_perm, (size_t)n * 4));
+    CU(dmalloc(g, &g->d_inv, (size_t)n * 4));
+    CU(dmalloc(g, &g->d_perm, (size_t)n * 4));
     int64_t maxlen = 0;
     for (int r = 0; r < g->p; ++r) maxlen = std::max(maxlen, g->part[r + 1] - g->part[r]);
     size_t tb = 0;
     CU(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, v0, g->d_inv, (int)maxlen, 0, 32, st));
     void *tmp = nullptr;
-    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    CU(dmalloc(g, &tmp, std::max<size_t>(tb, 16)));
     fr.p.push_back(tmp);
     for (int r = 0; r < g->p; ++r) {
         const int64_t b = g->part[r], len = g->part[r + 1] - b;
@@ -535,24 +565,24 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
 static atos_status relabel_rows(atos_graph *g, LocalRank &me) {
     cudaStream_t st = g->stream;
     const int64_t v0 = g->part[me.rank], nr = me.L.n_r;
-    DevFrees fr;
+    DevFrees fr(g);
     int64_t *deg = nullptr, *rp_new = nullptr;
     int32_t *col_new = nullptr;
-    CU(cudaMalloc(&deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
-    CU(cudaMalloc(&rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
-    CU(cudaMalloc(&col_new, (size_t)std::max<int64_t>(me.m_r, 1) * 4)); fr.p.push_back(col_new);
+    CU(dmalloc(g, &deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
+    CU(dmalloc(g, &rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
+    CU(dmalloc(g, &col_new, (size_t)std::max<int64_t>(me.m_r, 1) * 4)); fr.p.push_back(col_new);
     new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
     size_t tb = 0;
     CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
     void *tmp = nullptr;
-    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    CU(dmalloc(g, &tmp, std::max<size_t>(tb, 16)));
     fr.p.push_back(tmp);
     CU(cub::DeviceScan::ExclusiveSum(tmp, tb, deg, rp_new, (int64_t)(nr + 1), st));
     permute_rows_kernel<<<2048, 256, 0, st>>>(me.row_ptr, me.col, g->d_inv, g->d_perm, v0, nr, rp_new, col_new);
     CU(cudaGetLastError());
     CU(cudaStreamSynchronize(st));
-    cudaFree(me.row_ptr);
-    cudaFree(me.col);
+    dfree(g, me.row_ptr);
+    dfree(g, me.col);
     me.row_ptr = rp_new;
     me.col = col_new;
     fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)rp_new), fr.p.end());
@@ -570,24 +600,24 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
     cudaStream_t st = g->stream;
     const int r = me.rank;
     const int64_t v0 = g->part[r], nr = me.L.n_r, m = me.m_r, base = rp_host[v0];
-    DevFrees fr;
+    DevFrees fr(g);
     int64_t *deg = nullptr, *rp_new = nullptr;
     int32_t *col_new = nullptr;
-    CU(cudaMalloc(&deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
-    CU(cudaMalloc(&rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
-    CU(cudaMalloc(&col_new, (size_t)std::max<int64_t>(m, 1) * 4)); fr.p.push_back(col_new);
+    CU(dmalloc(g, &deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
+    CU(dmalloc(g, &rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
+    CU(dmalloc(g, &col_new, (size_t)std::max<int64_t>(m, 1) * 4)); fr.p.push_back(col_new);
     new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
     size_t tb = 0;
     CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
     void *tmp = nullptr;
-    CU(cudaMalloc(&tmp, std::max<size_t>(tb, 16)));
+    CU(dmalloc(g, &tmp, std::max<size_t>(tb, 16)));
     fr.p.push_back(tmp);
     CU(cub::DeviceScan::ExclusiveSum(tmp, tb, deg, rp_new, (int64_t)(nr + 1), st));
     int64_t ch = (int64_t)1 << 26;                  // 256 MB per stage
     if (const char *e = std::getenv("ATOS_LOAD_CHUNK")) ch = std::max<int64_t>(1, std::atoll(e));   // tests: many chunks
     const int64_t CH = std::min<int64_t>(std::max<int64_t>(m, 1), ch);
     int32_t *stage[2] = {nullptr, nullptr};
-    for (int k = 0; k < 2; ++k) { CU(cudaMalloc(&stage[k], (size_t)CH * 4)); fr.p.push_back(stage[k]); }
+    for (int k = 0; k < 2; ++k) { CU(dmalloc(g, &stage[k], (size_t)CH * 4)); fr.p.push_back(stage[k]); }
     cudaStream_t cs = nullptr;
     CU(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
     cudaEvent_t ev_in[2], ev_out[2], ev_ready;
@@ -642,7 +672,7 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
     cudaStreamDestroy(cs);
     if (status != ATOS_OK) return status;
     if (e != cudaSuccess) return fail(ATOS_ERR_CUDA, "streamed relabel: %s", cudaGetErrorString(e));
-    cudaFree(me.row_ptr);
+    dfree(g, me.row_ptr);
     me.row_ptr = rp_new;
     me.col = col_new;
     fr.p.erase(std::remove(fr.p.begin(), fr.p.end(), (void *)rp_new), fr.p.end());
@@ -738,6 +768,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         CU(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
         g->own_stream = true;
     }
+    pool_setup(cfg.device);
     CU(cudaEventCreate(&g->ev_begin));
     CU(cudaEventCreate(&g->ev_w0));
     CU(cudaEventCreate(&g->ev_w1));
@@ -761,14 +792,16 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         me.L = make_layout(g->S, g->part.data(), r);
         const int64_t nr = me.L.n_r;
         me.m_r = rb[r + 1] - rb[r];
-        CU(cudaMalloc(&me.arena, me.L.total));
+        if (g->multiproc) CU(cudaMalloc(&me.arena, me.L.total));   // IPC-exported
+        else CU(dmalloc(g, &me.arena, me.L.total));
         CU(cudaMemsetAsync(me.arena, 0, me.L.total, g->stream));
         tr.mark(g->stream, "arena");
         // host CSR + relabeling: stream the columns through the permutation (no
         // full-size device copy of the unpermuted columns)
-        const bool streamed = g->d_perm && me.m_r > 0 && !rp_dev && !is_device_ptr(col);
-        CU(cudaMalloc(&me.row_ptr, (size_t)(nr + 1) * 8));
-        if (!streamed) CU(cudaMalloc(&me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
+        const char *se = std::getenv("ATOS_LOAD_STREAMED");
+        const bool streamed = g->d_perm && me.m_r > 0 && !rp_dev && !is_device_ptr(col) && !(se && se[0] == '0');
+        CU(dmalloc(g, &me.row_ptr, (size_t)(nr + 1) * 8));
+        if (!streamed) CU(dmalloc(g, &me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
         CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
         if (me.m_r > 0 && !streamed)
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
@@ -807,7 +840,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (bad & 2) return fail(ATOS_ERR_INVALID_ARG, "csr: column index out of [0, n)");
 
     CU(cudaMalloc(&g->d_ranks, sizeof(RankDev) * g->n_local));
-    CU(cudaMalloc(&g->d_depth_full, (size_t)n * 4));
+    CU(dmalloc(g, &g->d_depth_full, (size_t)n * 4));
     CU(cudaMalloc(&g->d_accs, sizeof(int64_t *) * kMaxRanks));
     g->connected = !g->multiproc;
     atos_status st = upload_views(g);

@@ -50,7 +50,7 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
         R.ctrl->ring_base.v = R.ctrl->tail.v;
         if (src < R.v_begin || src >= R.v_end) continue;
         R.depth[src] = dw_make(0);
-        R.filt[src] = 0;
+        filt_put_fresh(R.filt, src, 0u);
         const uint64_t idx = R.ctrl->tail.v;
         uint64_t *p = &R.ring[idx & (R.ring_cap - 1)];
         if (!slot_free_for(*p, idx)) { R.ctrl->error.v = kErrCapacity; return; }

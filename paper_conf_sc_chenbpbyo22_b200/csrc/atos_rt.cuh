@@ -42,6 +42,33 @@ __device__ __forceinline__ uint32_t ldg_u8(const uint8_t *p) {
 __device__ __forceinline__ void stg_u8(uint8_t *p, uint32_t x) {
     asm volatile("st.global.u8 [%0], %1;" ::"l"(p), "h"((uint16_t)x));
 }
+// Filter access.  Default: one byte per vertex.  ATOS_FILTER4 (experiment): one
+// nibble per vertex (bound saturated at 15), half the footprint; the update is a
+// racy read-modify-write of the byte, which can only leave an older -- still
+// valid, larger -- bound in either nibble.  filt_probe returns the raw byte.
+#ifndef ATOS_FILTER4
+#define ATOS_FILTER4 0
+#endif
+__device__ __forceinline__ uint32_t filt_probe(const uint8_t *f, int64_t u) { return ldg_u8(f + (ATOS_FILTER4 ? (u >> 1) : u)); }
+__device__ __forceinline__ uint32_t filt_val(uint32_t raw, int64_t u) {
+    return ATOS_FILTER4 ? (raw >> ((u & 1) * 4)) & 15u : raw;
+}
+__device__ __forceinline__ bool filt_pass(uint32_t raw, int64_t u, uint32_t nd) {
+    const uint32_t fv = filt_val(raw, u);
+    return nd < fv || fv == (ATOS_FILTER4 ? 15u : 255u);
+}
+__device__ __forceinline__ void filt_put(uint8_t *f, int64_t u, uint32_t nd, uint32_t raw) {
+    if (ATOS_FILTER4) {
+        const int sh = (int)(u & 1) * 4;
+        const uint32_t x = nd < 15u ? nd : 15u;
+        stg_u8(f + (u >> 1), (raw & ~(15u << sh) & 0xFFu) | (x << sh));
+    } else {
+        stg_u8(f + u, filt_of(nd));
+    }
+}
+__device__ __forceinline__ void filt_put_fresh(uint8_t *f, int64_t u, uint32_t nd) {
+    filt_put(f, u, nd, ATOS_FILTER4 ? ldg_u8(f + (u >> 1)) : 0u);
+}
 
 #ifndef ATOS_THREADS
 #define ATOS_THREADS 512

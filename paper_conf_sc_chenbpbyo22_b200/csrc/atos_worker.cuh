@@ -485,7 +485,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                         if (i < cq) {
                             const uint32_t ndw = dw_make(hi32(m[j]));
                             pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
-                            if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(m[j])));
+                            if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(m[j]));
                         }
                     }
                 } else {
@@ -604,7 +604,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                     ul[j] = lo32(msg);
                     const uint32_t ndw = dw_make(hi32(msg));
                     pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
-                    if (pred[j] && kp.filter) stg_u8(R.filt + R.v_begin + ul[j], filt_of(hi32(msg)));
+                    if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(msg));
                 } else {
                     const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
                     ul[j] = msg.x;
@@ -669,7 +669,7 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
     uint32_t cur[N];
     if (fl) {
 #pragma unroll
-        for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? ldg_u8(filt + u[k]) : 0u;       // probe the filter
+        for (int k = 0; k < N; ++k) cur[k] = (u[k] >= 0) ? filt_probe(filt, u[k]) : 0u;     // probe the filter
     } else {
 #pragma unroll
         for (int k = 0; k < N; ++k) {
@@ -687,10 +687,10 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
 #pragma unroll
         for (int k = 0; k < N; ++k) {
             const uint32_t ndw = dw_make(nd[k]);
-            imp[k] = u[k] >= 0 && (fl ? filt_maybe(cur[k], nd[k]) : ndw < cur[k]);
+            imp[k] = u[k] >= 0 && (fl ? filt_pass(cur[k], u[k], nd[k]) : ndw < cur[k]);
             if (imp[k]) {
                 red_min_u32(depth + u[k], ndw);
-                if (fl) stg_u8(filt + u[k], filt_of(nd[k]));
+                if (fl) filt_put(filt, u[k], nd[k], cur[k]);
             }
         }
     } else {
@@ -698,9 +698,9 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
         for (int k = 0; k < N; ++k) {
             const uint32_t ndw = dw_make(nd[k]);
             imp[k] = false;
-            if (u[k] >= 0 && (fl ? filt_maybe(cur[k], nd[k]) : ndw < cur[k])) {
+            if (u[k] >= 0 && (fl ? filt_pass(cur[k], u[k], nd[k]) : ndw < cur[k])) {
                 imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
-                if (fl && imp[k]) stg_u8(filt + u[k], filt_of(nd[k]));
+                if (fl && imp[k]) filt_put(filt, u[k], nd[k], cur[k]);
             }
         }
     }
@@ -709,7 +709,7 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
 #pragma unroll
         for (int k = 0; k < N; ++k) {
             if (hs[k] >= 0) {
-                const uint32_t ob = fl ? cur[k] : dw_depth(cur[k]);
+                const uint32_t ob = fl ? filt_val(cur[k], u[k]) : dw_depth(cur[k]);
                 hub_put(hc, hs[k], ob < nd[k] ? ob : nd[k]);
             }
         }
@@ -755,18 +755,25 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
         int32_t u[kU];
         using ValT = typename std::conditional<APP == kApBfs, uint32_t, uint64_t>::type;   // depth | delta bits
         ValT vv[kU];
+        // the lane's current vertex in registers: column base (beg - off), value and the
+        // next vertex's first edge; shared memory is read again only when a row ends
+        int64_t cbase = bb.beg[j] - bb.off[j], nxt = j < jhi ? bb.off[j + 1] : INT64_MAX;
+        ValT cval = (ValT)bb.val[j];
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
             const int64_t e = c0 + k * 32 + lane;
             u[k] = -1;
             vv[k] = 0;
             if (e <= clast) {
-                if (j < jhi && bb.off[j + 1] <= e) {       // usually one step for skewed graphs
+                if (e >= nxt) {                             // usually one step for skewed graphs
                     ++j;
                     if (j < jhi && bb.off[j + 1] <= e) j = upper_vertex(bb, j + 1, jhi, e);
+                    cbase = bb.beg[j] - bb.off[j];
+                    nxt = j < jhi ? bb.off[j + 1] : INT64_MAX;
+                    cval = (ValT)bb.val[j];
                 }
-                u[k] = ld_stream(col + bb.beg[j] + (e - bb.off[j]), pol);
-                vv[k] = (ValT)bb.val[j];
+                u[k] = ld_stream(col + cbase + e, pol);
+                vv[k] = cval;
             }
         }
 #ifdef ATOS_PROF
@@ -972,7 +979,7 @@ __device__ __forceinline__ void probe_issue(const KParams &kp, const RankDev &R,
                                             uint32_t (&cur)[kPU]) {
 #pragma unroll
     for (int k = 0; k < kPU; ++k)
-        cur[k] = st.u[k] < 0 ? 0u : (kp.filter ? ldg_u8(R.filt + st.u[k]) : ldg_u32(R.depth + st.u[k]));
+        cur[k] = st.u[k] < 0 ? 0u : (kp.filter ? filt_probe(R.filt, st.u[k]) : ldg_u32(R.depth + st.u[k]));
 }
 
 template <int APP, bool MULTI>
@@ -986,7 +993,7 @@ __device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta
 #pragma unroll
     for (int k = 0; k < kPU; ++k) {
         const uint32_t nd = st.nd[k], ndw = dw_make(nd);
-        const bool maybe = st.u[k] >= 0 && (fl ? filt_maybe(cur[k], nd) : ndw < cur[k]);
+        const bool maybe = st.u[k] >= 0 && (fl ? filt_pass(cur[k], st.u[k], nd) : ndw < cur[k]);
         imp[k] = false;
         if (maybe) {
             if (kp.relax_red) {
@@ -995,7 +1002,7 @@ __device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta
             } else {
                 imp[k] = atom_min_u32(R.depth + st.u[k], ndw) > ndw;
             }
-            if (fl && imp[k]) stg_u8(R.filt + st.u[k], filt_of(nd));
+            if (fl && imp[k]) filt_put(R.filt, st.u[k], nd, cur[k]);
         }
     }
     if constexpr (!MULTI) {
