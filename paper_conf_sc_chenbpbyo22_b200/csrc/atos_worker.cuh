@@ -546,54 +546,36 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
         const int nc = R.n_ranks * kp.nsub;
         const int start = (cta + (int)s.c_idle) % nc;
         int got = 0;
-        // phase 1: one lane per sub-channel reads its cursor and the header there
-        // (two round trips for all channels instead of two per channel)
-        for (int base = 0; base < nc && !got; base += 32) {
-            const int ci = base + lane;
-            int chl = -1;
-            uint64_t ccl = 0;
-            bool cand = false;
-            if (ci < nc) {
-                chl = (start + ci) % nc;
-                const int srl = chl / kp.nsub, skl = chl % kp.nsub;
-                if (srl != R.rank) {
-                    ccl = ld_relaxed_gpu(&R.ctrl->in_cursor[chl].v);
-                    const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[srl][sub_slot(kp, skl, ccl)]);
-                    cand = hi32(h) == lo32(ccl + 1);
-                }
+        for (int kk = 0; kk < nc && !got; ++kk) {
+            const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
+            if (sr == R.rank) continue;
+            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+            uint64_t cc = 0;
+            if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+            cc = __shfl_sync(kFull, cc, 0);
+            bool ready = false;
+            uint32_t cnt = 0;
+            if (lane < kClaim && (uint32_t)lane < cps) {
+                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
+                ready = hi32(h) == lo32(cc + lane + 1);
+                cnt = lo32(h);
             }
-            uint32_t cm = __ballot_sync(kFull, cand);
-            // phase 2: claim the ready prefix of the first candidate that can be won
-            while (cm != 0u && !got) {
-                const int L = __ffs(cm) - 1;
-                cm &= cm - 1u;
-                const int ch = __shfl_sync(kFull, chl, L), sr = ch / kp.nsub, sk = ch % kp.nsub;
-                const uint64_t cc = __shfl_sync(kFull, ccl, L);
-                unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
-                bool ready = false;
-                uint32_t cnt = 0;
-                if (lane < kClaim && (uint32_t)lane < cps) {
-                    const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
-                    ready = hi32(h) == lo32(cc + lane + 1);
-                    cnt = lo32(h);
-                }
-                const uint32_t nready = __ballot_sync(kFull, ready);
-                const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
-                if (r == 0) continue;
-                int won = 0;
-                if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
-                if (!__shfl_sync(kFull, won, 0)) continue;
-                if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // sync with each sender's release
-                uint32_t incl = lane < r ? cnt : 0u;
+            const uint32_t nready = __ballot_sync(kFull, ready);
+            const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
+            if (r == 0) continue;
+            int won = 0;
+            if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+            if (!__shfl_sync(kFull, won, 0)) continue;
+            if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // sync with each sender's release
+            uint32_t incl = lane < r ? cnt : 0u;
 #pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {
-                    const uint32_t y = __shfl_up_sync(kFull, incl, d);
-                    if (lane >= d) incl += y;
-                }
-                if (lane < r) s.in_off[lane + 1] = incl;
-                if (lane == 0) { s.in_off[0] = 0; s.in_src = ch; s.in_cc = cc; s.in_r = r; }
-                got = 1;
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, d);
+                if (lane >= d) incl += y;
             }
+            if (lane < r) s.in_off[lane + 1] = incl;
+            if (lane == 0) { s.in_off[0] = 0; s.in_src = ch; s.in_cc = cc; s.in_r = r; }
+            got = 1;
         }
         if (lane == 0) s.in_got = got;
     }
