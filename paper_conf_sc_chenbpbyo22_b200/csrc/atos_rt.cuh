@@ -300,7 +300,8 @@ struct KParams {
     int32_t combine;         // PR sender-side residual combining (multi-rank)
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained
     int32_t sys;             // peers are other devices/processes: system-scope ordering (else .gpu)
-    int32_t early;           // reserve the next batch during expansion; per-warp enqueue (no keeping)
+    int32_t early;           // reserve the next batch during expansion
+    int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

@@ -1176,7 +1176,7 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         else expand_warp<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         // without work keeping, each warp enqueues its discoveries as soon as its
         // chunks are done (one atomic per warp) instead of after the batch barrier
-        if (kp.keep == 0 && kp.early) warp_flush_local(s, w, wn, APP == kApBfs && kp.relax_red);
+        if (kp.keep == 0 && kp.warp_flush) warp_flush_local(s, w, wn, APP == kApBfs && kp.relax_red);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
