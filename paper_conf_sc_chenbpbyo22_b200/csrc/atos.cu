@@ -921,7 +921,8 @@ static KParams make_params(atos_graph *g) {
     // early next-batch reservation + per-warp enqueue: measured within noise
     // (RMAT-24/26 BFS, RMAT-20 PR); off unless ATOS_EARLY is set (experiment)
     kp.early = std::getenv("ATOS_EARLY") ? 1 : 0;
-    kp.warp_flush = std::getenv("ATOS_WARP_FLUSH") ? 1 : 0;   // experiment   // virtual ranks share this device: .gpu scope suffices
+    kp.warp_flush = std::getenv("ATOS_WARP_FLUSH") ? 1 : 0;   // experiment
+    kp.edge_map = std::getenv("ATOS_NO_EDGE_MAP") ? 0 : 1;     // A/B switch   // virtual ranks share this device: .gpu scope suffices
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;

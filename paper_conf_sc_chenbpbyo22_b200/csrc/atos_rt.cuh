@@ -302,6 +302,7 @@ struct KParams {
     int32_t sys;             // peers are other devices/processes: system-scope ordering (else .gpu)
     int32_t early;           // reserve the next batch during expansion
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
+    int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

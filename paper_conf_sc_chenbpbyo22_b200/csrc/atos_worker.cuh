@@ -73,6 +73,14 @@ template <> struct AppTraits<kApBfs> { static constexpr int kMsgBytes = 8; };
 template <> struct AppTraits<kApPr> { static constexpr int kMsgBytes = 16; };
 
 // One popped batch, set up for expansion.
+// Edge -> vertex map of a batch with E <= kBitE edges (DESIGN.md 5.1 "edge map"):
+// bit e of bm marks the first edge of a non-empty row, rowmap[w] is the (compacted)
+// row holding edge 32w, nzslot[] maps compacted rows to batch slots.  A lane's row
+// is then rowmap[w] + popc(bm[w] & lanes (0, lane]) -- one word per 32 edges
+// instead of a per-lane binary search over the batch offsets.
+constexpr int kBitW = 2048;
+constexpr int64_t kBitE = (int64_t)kBitW * 32;
+
 struct BatchBuf {
     uint32_t v[kThreads];          // local vertex ids
     uint64_t val[kThreads];        // depth (BFS) or delta bits (PR)
@@ -80,7 +88,18 @@ struct BatchBuf {
     int64_t off[kThreads + 1];     // exclusive prefix of edge counts
     uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
     uint32_t chunk_next;           // next unclaimed edge chunk
+    int32_t use_bm;                // the edge map below is valid for this batch
+    uint32_t bm[kBitW];
+    uint16_t rowmap[kBitW];
+    uint16_t nzslot[kThreads];
 };
+
+// batch slot holding edge e (e = 32 * w + lane) from the edge map
+__device__ __forceinline__ int bm_slot(const BatchBuf &bb, int64_t e, int lane) {
+    const int w = (int)(e >> 5);
+    const uint32_t below = lane == 31 ? 0xFFFFFFFEu : (((2u << lane) - 1u) & ~1u);
+    return bb.nzslot[bb.rowmap[w] + __popc(bb.bm[w] & below)];
+}
 
 struct Smem {
     RankDev R;
@@ -751,10 +770,23 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
             jhi = upper_vertex(bb, jlo, B - 1, clast);
         }
         jprev = jlo;
-        int j = jlo;
         int32_t u[kU];
         using ValT = typename std::conditional<APP == kApBfs, uint32_t, uint64_t>::type;   // depth | delta bits
         ValT vv[kU];
+        if (bb.use_bm) {
+#pragma unroll
+            for (int k = 0; k < kU; ++k) {
+                const int64_t e = c0 + k * 32 + lane;
+                u[k] = -1;
+                vv[k] = 0;
+                if (e <= clast) {
+                    const int jj = bm_slot(bb, e, lane);
+                    u[k] = ld_stream(col + bb.beg[jj] + (e - bb.off[jj]), pol);
+                    vv[k] = (ValT)bb.val[jj];
+                }
+            }
+        } else {
+        int j = jlo;
         // the lane's current vertex in registers: column base (beg - off), value and the
         // next vertex's first edge; shared memory is read again only when a row ends
         int64_t cbase = bb.beg[j] - bb.off[j], nxt = j < jhi ? bb.off[j + 1] : INT64_MAX;
@@ -775,6 +807,7 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                 u[k] = ld_stream(col + cbase + e, pol);
                 vv[k] = cval;
             }
+        }
         }
 #ifdef ATOS_PROF
         { int32_t sk = 0; for (int k = 0; k < kU; ++k) sk |= u[k]; PROF_T(pt1, sk); }
@@ -895,6 +928,20 @@ __device__ __forceinline__ void pipe_load(const BatchBuf &bb, int B, int64_t E, 
     const int lane = threadIdx.x & 31;
     const int64_t c0 = (int64_t)c * kPChunk;
     const int64_t clast = (E < c0 + kPChunk ? E : c0 + kPChunk) - 1;
+    if (bb.use_bm) {
+#pragma unroll
+        for (int k = 0; k < kPU; ++k) {
+            const int64_t e = c0 + k * 32 + lane;
+            st.u[k] = -1;
+            st.nd[k] = 0;
+            if (e <= clast) {
+                const int jj = bm_slot(bb, e, lane);
+                st.u[k] = ld_stream(col + bb.beg[jj] + (e - bb.off[jj]), pol);
+                st.nd[k] = (uint32_t)bb.val[jj] + 1u;
+            }
+        }
+        return;
+    }
     const uint32_t m = (uint32_t)(c0 / kChunk);          // map chunk containing c0
     int jlo, jhi;
     if (m + 1 < (uint32_t)kChunkMap) {
@@ -1134,16 +1181,27 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
             ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
     }
     if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + bb.beg[tid], (uint64_t)deg * 4);
-    int64_t excl;
-    const int64_t E = block_exscan(s, deg, excl);
+    if (kp.edge_map)
+        for (int i = tid; i < kBitW; i += kThreads) bb.bm[i] = 0u;   // ordered before the map by the scan's barriers
+    // one scan for both the edge offsets and the compacted index of non-empty rows
+    int64_t pexcl;
+    const int64_t ptot = block_exscan(s, (deg << 16) | (deg > 0 ? 1 : 0), pexcl);
+    const int64_t excl = pexcl >> 16, E = ptot >> 16;
+    const bool use_bm = kp.edge_map && E <= kBitE;
     if (tid < B) {
         bb.off[tid] = excl;
         if (deg > 0) {   // chunk -> first vertex map: chunks starting inside this row
             const int64_t cl = (excl + deg - 1) / kChunk;
             for (int64_t c = (excl + kChunk - 1) / kChunk; c <= cl && c < kChunkMap; ++c) bb.chunk_v[c] = (uint16_t)tid;
+            if (use_bm) {
+                const int nz = (int)(pexcl & 0xFFFF);
+                bb.nzslot[nz] = (uint16_t)tid;
+                atomicOr(&bb.bm[excl >> 5], 1u << (excl & 31));
+                for (int64_t w = (excl + 31) >> 5; w <= ((excl + deg - 1) >> 5); ++w) bb.rowmap[w] = (uint16_t)nz;
+            }
         }
     }
-    if (tid == 0) { bb.off[B] = E; s.c_edges += (unsigned long long)E; bb.chunk_next = 0; }
+    if (tid == 0) { bb.off[B] = E; s.c_edges += (unsigned long long)E; bb.chunk_next = 0; bb.use_bm = use_bm ? 1 : 0; }
     __syncthreads();
 #ifdef ATOS_PROF
     if (tid == 0) s.prof[7] += (unsigned long long)clock64();   // minus entry below: setup+scan
