@@ -303,6 +303,7 @@ struct KParams {
     int32_t early;           // reserve the next batch during expansion
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
+    int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

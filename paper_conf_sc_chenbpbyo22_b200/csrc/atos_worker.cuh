@@ -750,11 +750,17 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
     const uint64_t pol = policy_evict_first();
     const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
     int jprev = 0;
+    uint32_t cs = (uint32_t)(threadIdx.x >> 5);   // static schedule: chunks w, w + 16, ...
     for (;;) {
-        // dynamic chunk claim: a warp that finishes early takes the next chunk
         uint32_t c = 0;
-        if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
-        c = __shfl_sync(kFull, c, 0);
+        if (kp.static_chunks) {
+            c = cs;
+            cs += kWarps;
+        } else {
+            // dynamic chunk claim: a warp that finishes early takes the next chunk
+            if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
+            c = __shfl_sync(kFull, c, 0);
+        }
         if (c >= nch) break;
 #ifdef ATOS_PROF
         long long pt0 = clock64(), pt1, pt2, pt3, pt4;
