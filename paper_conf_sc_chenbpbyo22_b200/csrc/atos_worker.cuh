@@ -750,18 +750,15 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
     const uint64_t pol = policy_evict_first();
     const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
     int jprev = 0;
-    // the first 3/4 of the chunks are dealt round-robin (chunk w, w + 16, ...: no
-    // claim per chunk), the rest are claimed dynamically so that warps whose chunks
-    // missed L2 more often do not hold up the batch barrier
-    const uint32_t nstat = kp.static_chunks ? (nch - nch / 4) : 0u;
-    uint32_t cs = (uint32_t)(threadIdx.x >> 5);
+    uint32_t cs = (uint32_t)(threadIdx.x >> 5);   // static schedule: chunks w, w + 16, ...
     for (;;) {
         uint32_t c = 0;
-        if (cs < nstat) {
+        if (kp.static_chunks) {
             c = cs;
             cs += kWarps;
         } else {
-            if (lane == 0) c = nstat + atomicAdd(&bb.chunk_next, 1u);
+            // dynamic chunk claim: a warp that finishes early takes the next chunk
+            if (lane == 0) c = atomicAdd(&bb.chunk_next, 1u);
             c = __shfl_sync(kFull, c, 0);
         }
         if (c >= nch) break;
@@ -1375,9 +1372,7 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
         bb.v[tid] = lo32(slot);
         st_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)], pack(lo32(idx + R.ring_cap), 0u));
     }
-    // no barrier here: bb.v[t] is read next by thread t itself, every thread read
-    // s.res_lo before the barrier above, and a barrier always separates this from
-    // the next pop (process_batch's scan, or the loop head when B == 0)
+    __syncthreads();
     if (tid == 0) s.res_lo = lo + (uint64_t)B;
     return B;
 }
