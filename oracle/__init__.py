@@ -7,7 +7,8 @@ Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
 Functions (see oracle.c for the paper passages each one follows):
   bfs(row_ptr, col, src)                -> depth int32 [n]   (-1 = unreachable)
   bfs_parents_minid(row_ptr, col, depth, src) -> parent int64 [n]
-  pagerank(row_ptr, col, alpha, tol)    -> (p float64 [n] with sum 1, iterations, final L1 delta)
+  pagerank(row_ptr, col, alpha, tol)    -> (p float64 [n] with sum 1, iterations, final L1 delta);
+                                           raises RuntimeError if max_iter ends before ||dp||_1 <= tol
 
 Parity status: BFS pinned (brute force / closed forms / scipy); PageRank pinned
 (closed forms / dense solve / networkx).  See tests/test_oracle.py.
@@ -101,6 +102,9 @@ def pagerank(row_ptr, col, alpha: float = 0.85, tol: float = 1e-12, max_iter: in
     delta = ctypes.c_double(0.0)
     rc = _load().oracle_pagerank(n, _ptr(rp), _ptr(c), float(alpha), float(tol), int(max_iter),
                                  int(nthreads), _ptr(p), ctypes.byref(it), ctypes.byref(delta))
+    if rc == 4:
+        raise RuntimeError(f"oracle_pagerank did not converge: ||dp||_1 = {delta.value:.3e} > tol {tol:.1e} "
+                           f"after {it.value} iterations (max_iter {max_iter})")
     if rc != 0:
         raise ValueError(f"oracle_pagerank failed rc={rc}")
     return p, it.value, delta.value

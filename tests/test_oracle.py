@@ -272,3 +272,15 @@ def test_pr_thread_count_invariant():
     p1, it1, _ = oracle.pagerank(rp, col, 0.85, nthreads=1)
     p4, it4, _ = oracle.pagerank(rp, col, 0.85, nthreads=4)
     assert it1 == it4 and np.array_equal(p1, p4)
+
+
+def test_pr_not_converged_is_an_error():
+    """The oracle's answer is the fixed point to ||dp||_1 <= tol (north_star: Jacobi
+    iterated to a 1e-12 L1 residual); a run cut off by max_iter must not silently
+    become an expected value."""
+    g = inputs.rmat(10, 16, 3, symmetric=False)
+    rp, col = g.numpy()
+    with pytest.raises(RuntimeError, match="did not converge"):
+        oracle.pagerank(rp, col, 0.85, tol=1e-12, max_iter=3)
+    p, it, delta = oracle.pagerank(rp, col, 0.85, tol=1e-12)
+    assert delta <= 1e-12 and it > 3
