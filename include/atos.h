@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define ATOS_ABI_VERSION 3
+#define ATOS_ABI_VERSION 4
 #define ATOS_MAX_RANKS 8          /* one NVSwitch box: 8 GPUs */
 #define ATOS_IPC_HANDLE_BYTES 64  /* == sizeof(cudaIpcMemHandle_t) */
 
@@ -137,6 +137,11 @@ typedef struct {
                                  ghost mass (< eps in total per vertex beyond
                                  the owner's own < eps).  0 = send every delta
                                  (the paper's push, with aggregation)          */
+    int32_t pool_retain;      /* 0 = atos_graph_free trims the library's private
+                                 stream-ordered memory pool back to zero (freed
+                                 memory returns to the device); 1 = keep it
+                                 reserved for the next graph_load in this
+                                 process (load/solve/free loops)               */
 } atos_config;
 
 /* Per-solve statistics (device counters, summed over the ranks this handle
@@ -213,7 +218,14 @@ atos_status atos_bfs(atos_graph *g, int64_t src, int32_t *depth_out, int64_t *pa
 atos_status atos_pagerank(atos_graph *g, double alpha, double eps, double *rank_out,
                           double *residual_out, atos_stats *stats);
 
-/* Wait for the last enqueued solve and return its device status. */
+/* Set the device watchdog of later solves (ms; 0 = none).  Host only. */
+atos_status atos_set_watchdog(atos_graph *g, int64_t ms);
+
+/* Wait for the last enqueued solve and return its device status.
+ * After a device error (ATOS_ERR_CAPACITY / ATOS_ERR_TIMEOUT) the outputs of
+ * that solve are invalid; a single-process handle (n_ranks == 1, any
+ * virtual_ranks) is reset to its just-loaded state and can solve again, a
+ * multi-process handle is poisoned: later solves return ATOS_ERR_STATE. */
 atos_status atos_sync(atos_graph *g);
 
 /* Counters of the last completed solve (synchronises). */

@@ -36,6 +36,19 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS if os.path.exists(d))
 
 
+def variant() -> bool:
+    """An experiment variant library was requested (ATOS_LIB)."""
+    return bool(os.environ.get("ATOS_LIB"))
+
+
+def source_commit() -> str:
+    try:
+        return subprocess.check_output(["git", "-C", ROOT, "rev-parse", "--short=12", "HEAD"],
+                                       stderr=subprocess.DEVNULL, text=True).strip()
+    except Exception:
+        return "unknown"
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
@@ -44,6 +57,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
     cmd = [nvcc()] + NVCC_FLAGS + extra + (["-Xptxas", "-v"] if verbose else []) + ["-o", tmp] + SOURCES
     subprocess.check_call(cmd)
     os.replace(tmp, LIB)
+    # provenance beside every built library (A/B variants must say what they are)
+    dirty = ""
+    try:
+        if subprocess.check_output(["git", "-C", ROOT, "status", "--porcelain", "--", "paper_conf_sc_chenbpbyo22_b200/csrc",
+                                    "include"], stderr=subprocess.DEVNULL, text=True).strip():
+            dirty = " (sources modified after this commit)"
+    except Exception:
+        pass
+    with open(LIB + ".info", "w") as f:
+        f.write(f"commit {source_commit()}{dirty}\nATOS_NVCC_EXTRA={' '.join(extra)}\n")
     return LIB
 
 

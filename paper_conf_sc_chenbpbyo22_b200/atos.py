@@ -55,6 +55,7 @@ class Config(ctypes.Structure):
         ("keep_mode", ctypes.c_int32),
         ("discrete", ctypes.c_int32),
         ("pr_combine", ctypes.c_int32),
+        ("pool_retain", ctypes.c_int32),
     ]
 
 
@@ -103,6 +104,7 @@ _SIGS = [
     ("atos_graph_connect", ctypes.c_int, [_P, _P]),
     ("atos_bfs", ctypes.c_int, [_P, ctypes.c_int64, _P, _P, ctypes.POINTER(Stats)]),
     ("atos_pagerank", ctypes.c_int, [_P, ctypes.c_double, ctypes.c_double, _P, _P, ctypes.POINTER(Stats)]),
+    ("atos_set_watchdog", ctypes.c_int, [_P, ctypes.c_int64]),
     ("atos_sync", ctypes.c_int, [_P]),
     ("atos_last_stats", ctypes.c_int, [_P, ctypes.POINTER(Stats)]),
     ("atos_graph_free", ctypes.c_int, [_P]),
@@ -121,7 +123,12 @@ def load(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_build.LIB) or _build.stale():
+    if _build.variant():
+        # an A/B variant is used exactly as built (never silently rebuilt from the
+        # current tree, which could make two arms run identical code)
+        if not os.path.exists(_build.LIB):
+            raise FileNotFoundError(f"ATOS_LIB={_build.LIB} does not exist (build it with ATOS_NVCC_EXTRA first)")
+    elif not os.path.exists(_build.LIB) or _build.stale():
         if not build_if_missing:
             raise FileNotFoundError(f"{_build.LIB} missing; run __graft_entry__.build()")
         _build.build()
@@ -244,6 +251,9 @@ class Graph:
         if st is not None:
             return rank_out, residual_out, st.as_dict()
         return rank_out, residual_out
+
+    def set_watchdog(self, ms: int):
+        _check(self._lib.atos_set_watchdog(self._h, int(ms)))
 
     def sync(self):
         _check(self._lib.atos_sync(self._h))

@@ -94,6 +94,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->hub_cache = -1;
     cfg->split_edges = -1;
     cfg->pr_combine = 0;
+    cfg->pool_retain = 0;
     return ATOS_OK;
 }
 
@@ -129,7 +130,7 @@ static bool valid_cfg(const atos_config &c) {
            (c.hub_cache <= 0 || c.hub_cache % (32 * std::max(c.n_ranks, c.virtual_ranks)) == 0) &&
            (c.split_edges == 0 || c.split_edges == -1 ||
             (c.split_edges >= 256 && c.split_edges <= (1 << 20) && pow2(c.split_edges))) &&
-           (c.pr_combine == 0 || c.pr_combine == 1) &&
+           (c.pr_combine == 0 || c.pr_combine == 1) && (c.pool_retain == 0 || c.pool_retain == 1) &&
            (c.discrete == 0 || (c.discrete == 1 && c.n_ranks == 1 && c.virtual_ranks == 1));
 }
 
@@ -230,6 +231,7 @@ struct atos_graph {
     uint64_t epoch = 0;
     cudaEvent_t ev_begin = nullptr, ev_w0 = nullptr, ev_w1 = nullptr, ev_end = nullptr;
     bool pending = false;      // a solve is enqueued but not yet checked
+    bool poisoned = false;     // multi-process handle after a device error: no further solves
     int app = kApBfs;          // application of the pending / last solve
     atos_stats last{};
     bool last_valid = false;
@@ -240,27 +242,43 @@ struct atos_graph {
     cudaGraphExec_t dexec[2] = {nullptr, nullptr};
 };
 
-// Device memory of a handle comes from the device's default stream-ordered pool
-// with an unbounded release threshold, allocated and freed on the handle's
-// stream: a user loop that loads, solves and frees graphs (bench.py's e2e) reuses
-// physical memory instead of mapping and unmapping GBs through cudaMalloc /
-// cudaFree every time (measured 10-600 ms per call, varying).  The arena of a
-// multi-process handle stays on cudaMalloc: it is exported with cudaIpcGetMemHandle.
-static void pool_setup(int device) {
-    static bool done[64] = {false};
-    if (device < 0 || device >= 64 || done[device]) return;
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+// Device memory of a handle comes from a PRIVATE stream-ordered pool per device
+// (cudaMemPoolCreate; never the device's default pool, so no other library's
+// cudaMallocAsync is affected), allocated and freed on the handle's stream.  The
+// pool's release threshold is unbounded so that memory freed by one handle can be
+// reused by the next load in the same process without re-mapping (plain
+// cudaMalloc / cudaFree of GB buffers measured 10-600 ms per call);
+// atos_graph_free trims the pool back to zero unless cfg.pool_retain is set, so
+// by default a freed graph's memory goes back to the device (and to torch's
+// allocator).  The arena of a multi-process handle stays on cudaMalloc: it is
+// exported with cudaIpcGetMemHandle.
+#include <mutex>
+static cudaMemPool_t pool_of(int device) {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {nullptr};
+    if (device < 0 || device >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[device]) {
+        cudaMemPoolProps pr{};
+        pr.allocType = cudaMemAllocationTypePinned;
+        pr.location.type = cudaMemLocationTypeDevice;
+        pr.location.id = device;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &pr) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
         uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-        done[device] = true;
-    } else {
-        cudaGetLastError();
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[device] = p;
     }
+    return pools[device];
 }
 template <typename T>
 static cudaError_t dmalloc(const atos_graph *g, T **p, size_t bytes) {
-    return cudaMallocAsync((void **)p, bytes, g->stream);
+    cudaMemPool_t pool = pool_of(g->cfg.device);
+    if (!pool) return cudaMallocAsync((void **)p, bytes, g->stream);
+    return cudaMallocFromPoolAsync((void **)p, bytes, pool, g->stream);
 }
 static void dfree(const atos_graph *g, void *p) {
     if (p) cudaFreeAsync(p, g->stream);
@@ -449,10 +467,20 @@ static atos_status upload_views(atos_graph *g) {
     return ATOS_OK;
 }
 
+static KParams make_params(atos_graph *g);
+
 extern "C" atos_status atos_graph_free(atos_graph *g) {
     if (!g) return ATOS_OK;
     cudaSetDevice(g->cfg.device);
     if (g->stream) cudaStreamSynchronize(g->stream);
+    if (g->multiproc && g->connected && !g->poisoned && g->d_ranks) {
+        // peers may still be reading this rank's arena over NVLink (the gather and
+        // parent passes of the last solve): every rank arrives here before any
+        // rank unmaps or frees (epoch*4+2: above every barrier value of the solve)
+        KParams kp = make_params(g);
+        barrier_kernel<<<1, 32, 0, g->stream>>>(kp, g->epoch * 4 + 2);
+        cudaStreamSynchronize(g->stream);
+    }
     for (int s = 0; s < kMaxRanks; ++s)
         if (g->peer_opened[s]) cudaIpcCloseMemHandle(g->peer_base[s]);
     for (int lr = 0; lr < g->n_local; ++lr) {
@@ -477,6 +505,8 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     if (g->ev_w1) cudaEventDestroy(g->ev_w1);
     if (g->ev_end) cudaEventDestroy(g->ev_end);
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
+    if (!g->cfg.pool_retain)
+        if (cudaMemPool_t pool = pool_of(g->cfg.device)) cudaMemPoolTrimTo(pool, 0);   // freed memory back to the device
     delete g;
     return ATOS_OK;
 }
@@ -768,7 +798,6 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         CU(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
         g->own_stream = true;
     }
-    pool_setup(cfg.device);
     CU(cudaEventCreate(&g->ev_begin));
     CU(cudaEventCreate(&g->ev_w0));
     CU(cudaEventCreate(&g->ev_w1));
@@ -917,7 +946,7 @@ static KParams make_params(atos_graph *g) {
     kp.hc_per_rank = g->hc_per_rank;
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
-    kp.sys = g->multiproc ? 1 : 0;
+    kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
     // early next-batch reservation + per-warp enqueue: measured within noise
     // (RMAT-24/26 BFS, RMAT-20 PR); off unless ATOS_EARLY is set (experiment)
     kp.early = std::getenv("ATOS_EARLY") ? 1 : 0;
@@ -925,7 +954,9 @@ static KParams make_params(atos_graph *g) {
     kp.edge_map = std::getenv("ATOS_NO_EDGE_MAP") ? 0 : 1;     // A/B switch
     // round-robin chunks (no shared-memory claim per chunk): RMAT-24 3.06 -> 3.00 ms,
     // PR 12.65 -> 12.55 ms; ATOS_DYNAMIC_CHUNKS restores the claiming (A/B)
-    kp.static_chunks = std::getenv("ATOS_DYNAMIC_CHUNKS") ? 0 : 1;   // virtual ranks share this device: .gpu scope suffices
+    kp.static_chunks = std::getenv("ATOS_DYNAMIC_CHUNKS") ? 0 : 1;
+    if (const char *f = std::getenv("ATOS_TEST_FAULT"))   // test-only fault injection (T6 error paths)
+        kp.fault = std::strcmp(f, "capacity") == 0 ? kFaultCapacity : std::strcmp(f, "timeout") == 0 ? kFaultTimeout : 0;
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;
@@ -1057,6 +1088,24 @@ static atos_status read_ctrl(atos_graph *g, int lr, Ctrl &c) {
 // Wait for the enqueued solve, check device error flags, fill g->last.
 static constexpr int kSnap = 10;
 
+// Back to the state graph_load left: control blocks, rings, channel headers and
+// free mirrors re-initialised, statistics snapshots cleared.  Single process only.
+static atos_status reset_queues(atos_graph *g) {
+    for (int lr = 0; lr < g->n_local; ++lr) {
+        LocalRank &me = g->loc[lr];
+        CU(cudaMemsetAsync(me.arena + me.L.ctrl, 0, sizeof(Ctrl), g->stream));
+        CU(cudaMemsetAsync(me.arena + me.L.in_hdr, 0, me.L.in_pay - me.L.in_hdr, g->stream));
+        const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
+        init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
+                                                       (uint64_t *)(me.arena + me.L.free_m), nfree,
+                                                       (uint64_t)(g->S.cp / nsub_for(g->p, g->S.cp)));
+        CU(cudaGetLastError());
+        std::memset(me.snap, 0, sizeof(me.snap));
+    }
+    CU(cudaStreamSynchronize(g->stream));
+    return ATOS_OK;
+}
+
 static atos_status finish_solve(atos_graph *g) {
     const int app = g->app;
     if (!g->pending) return ATOS_OK;
@@ -1096,10 +1145,28 @@ static atos_status finish_solve(atos_graph *g) {
                                                             : AppTraits<kApPr>::kMsgBytes);
     g->last = st;
     g->last_valid = true;
+    if (err) {
+        // The aborted solve left reserved-but-unconsumed ring slots, channel packets
+        // and S/R/F/T counters that no later solve could reconcile.  A handle that
+        // owns every rank (single rank or virtual ranks) is reset to its
+        // just-loaded state; a multi-process handle cannot reset its peers' view of
+        // the channels alone, so it is poisoned (later solves: ATOS_ERR_STATE).
+        if (g->multiproc) g->poisoned = true;
+        else {
+            atos_status rs = reset_queues(g);
+            if (rs != ATOS_OK) return rs;
+        }
+    }
     if (err == kErrCapacity) return fail(ATOS_ERR_CAPACITY, "device queue/channel capacity exceeded; result invalid");
     if (err == kErrTimeout) return fail(ATOS_ERR_TIMEOUT, "device watchdog (%lld ms) fired; result invalid",
                                         (long long)g->cfg.watchdog_ms);
     if (err) return fail(ATOS_ERR_STATE, "device error %llu", (unsigned long long)err);
+    return ATOS_OK;
+}
+
+extern "C" atos_status atos_set_watchdog(atos_graph *g, int64_t ms) {
+    if (!g || ms < 0) return fail(ATOS_ERR_INVALID_ARG, "set_watchdog: NULL handle or ms < 0");
+    g->cfg.watchdog_ms = ms;
     return ATOS_OK;
 }
 
@@ -1121,6 +1188,7 @@ extern "C" atos_status atos_last_stats(atos_graph *g, atos_stats *stats) {
 static atos_status begin_solve(atos_graph *g, KParams &kp) {
     CU(cudaSetDevice(g->cfg.device));
     if (!g->connected) return fail(ATOS_ERR_PEER, "multi-process handle not connected (atos_graph_connect)");
+    if (g->poisoned) return fail(ATOS_ERR_STATE, "multi-process handle poisoned by an earlier device error; free and reload it");
     atos_status s = finish_solve(g);   // a previous async solve must be retired first
     if (s != ATOS_OK) return s;
     g->epoch++;
@@ -1174,14 +1242,14 @@ extern "C" atos_status atos_bfs(atos_graph *g, int64_t src, int32_t *depth_out, 
         int64_t *pout = parent_out;
         int64_t *ptmp = nullptr;
         if (!dev_parent) {
-            CU(cudaMallocAsync(&ptmp, (size_t)g->n * 8, g->stream));
+            CU(dmalloc(g, &ptmp, (size_t)g->n * 8));
             pout = ptmp;
         }
         parent_final_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(dfull, g->d_accs, n_acc, g->n,
                                                                                 src, pout);
         if (!dev_parent) {
             CU(cudaMemcpyAsync(parent_out, ptmp, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
-            CU(cudaFreeAsync(ptmp, g->stream));
+            dfree(g, ptmp);
         }
     }
     if (!dev_depth) CU(cudaMemcpyAsync(depth_out, dfull, (size_t)g->n * 4, cudaMemcpyDeviceToHost, g->stream));
@@ -1222,15 +1290,15 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     if (!dev_r || !dev_s) {
         // stage through the (idle) parent accumulator region: 8n bytes each is not
         // guaranteed, so use the full-depth buffer region only for one output.
-        CU(cudaMallocAsync(&tr, (size_t)g->n * 8, g->stream));
-        CU(cudaMallocAsync(&ts, (size_t)g->n * 8, g->stream));
+        CU(dmalloc(g, &tr, (size_t)g->n * 8));
+        CU(dmalloc(g, &ts, (size_t)g->n * 8));
     }
     gather_pr_kernel<<<grid_for(g->n, 512, gblocks), 512, 0, g->stream>>>(
         kp, rank_out ? (dev_r ? rank_out : tr) : nullptr, residual_out ? (dev_s ? residual_out : ts) : nullptr);
     if (rank_out && !dev_r) CU(cudaMemcpyAsync(rank_out, tr, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
     if (residual_out && !dev_s) CU(cudaMemcpyAsync(residual_out, ts, (size_t)g->n * 8, cudaMemcpyDeviceToHost, g->stream));
-    if (tr) CU(cudaFreeAsync(tr, g->stream));
-    if (ts) CU(cudaFreeAsync(ts, g->stream));
+    dfree(g, tr);
+    dfree(g, ts);
     CU(cudaGetLastError());
     CU(cudaEventRecord(g->ev_end, g->stream));
     g->pending = true;

@@ -218,6 +218,8 @@ struct alignas(128) Line {
 };
 
 enum DevError : uint64_t { kErrNone = 0, kErrCapacity = 4, kErrTimeout = 5 };
+// test-only fault injection (KParams::fault, env ATOS_TEST_FAULT): raise this error at worker start
+enum FaultKind : int32_t { kFaultNone = 0, kFaultCapacity = 1, kFaultTimeout = 2 };
 
 struct Ctrl {
     Line head;                   // local ring: next index to reserve for pop
@@ -304,6 +306,7 @@ struct KParams {
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming
+    int32_t fault;           // test-only fault injection (FaultKind), raised by rank 0 CTA 0 at start
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;
@@ -329,8 +332,15 @@ __device__ __forceinline__ int64_t pr_slot(int64_t i, int64_t q) {
     return (q > 0 && i < 8 * q) ? (i & 7) * q + (i >> 3) : i;
 }
 
+// Raise a device error for the current solve on this rank AND every peer, so
+// that all ranks' workers leave the loop (a rank that only waited for the
+// coordinator's done flag would otherwise spin until its own watchdog).  The
+// first code wins on each rank; system-scope CAS reaches IPC-mapped peers.
 __device__ __forceinline__ void set_error(const RankDev &R, uint64_t code) {
     atomicCAS((unsigned long long *)&R.ctrl->error.v, 0ull, (unsigned long long)code);
+    for (int d = 0; d < R.n_ranks && d < kMaxRanks; ++d)
+        if (d != R.rank && R.peer_ctrl[d])
+            atomicCAS_system((unsigned long long *)&R.peer_ctrl[d]->error.v, 0ull, (unsigned long long)code);
 }
 
 }  // namespace atos

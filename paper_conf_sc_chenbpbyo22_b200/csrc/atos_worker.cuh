@@ -1468,11 +1468,19 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
     const uint64_t t_start = globaltimer();
     uint32_t idle_streak = 0;
 
+    if (kp.fault && tid == 0 && cta == 0 && s.R.rank == 0)     // test-only fault injection (T6 error paths)
+        set_error(s.R, kp.fault == kFaultCapacity ? kErrCapacity : kErrTimeout);
     for (;;) {
         if (tid == 0) {
             int f = 0;
             if (ld_relaxed_gpu(&s.R.ctrl->done.v) == kp.epoch) f = 1;
             if (ld_relaxed_gpu(&s.R.ctrl->error.v) != 0) f = 2;
+            // the watchdog is checked on every iteration, busy or idle: a solve that
+            // never idles must still be stopped
+            if (kp.watchdog_ns > 0 && globaltimer() - t_start > (uint64_t)kp.watchdog_ns) {
+                set_error(s.R, kErrTimeout);
+                f = 2;
+            }
             s.flag = f;
         }
         __syncthreads();
@@ -1546,8 +1554,6 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
                 const uint64_t T = ld_acquire_gpu(&s.R.ctrl->tail.v);
                 if (F == T) st_release_gpu(&s.R.ctrl->done.v, kp.epoch);
             }
-            if (kp.watchdog_ns > 0 && globaltimer() - t_start > (uint64_t)kp.watchdog_ns)
-                set_error(s.R, kErrTimeout);
         }
         if (coordinator) coordinator_step(s, kp);
         if (idle_streak > 4) __nanosleep(idle_streak > 64 ? 256 : 32);

@@ -22,9 +22,10 @@ def main():
     rank, world, _ = adist.init(backend="gloo")
     torch.cuda.set_device(0)
     ok = True
-    g = inputs.rmat(13, 16, 1, symmetric=True)
+    scale = int(os.environ.get("ATOS_MP_SCALE", "13"))
+    g = inputs.rmat(scale, 16, 1, symmetric=True)
     rp, col = g.numpy()
-    G = atos.Graph(rp, col, g.n, rank=rank, n_ranks=world, device=0, ctas_per_sm=1, watchdog_ms=120000,
+    G = atos.Graph(rp, col, g.n, rank=rank, n_ranks=world, device=0, ctas_per_sm=1, watchdog_ms=600000,
                    channel_packets=64)
     adist.connect_graph(G, world)
     dist.barrier()
@@ -37,9 +38,9 @@ def main():
               f"packets={st['packets_sent']} ms={st['ms_worker']:.1f}", flush=True)
         dist.barrier()
     G.free()
-    gd = inputs.rmat(12, 16, 2, symmetric=False)
+    gd = inputs.rmat(scale - 1, 16, 2, symmetric=False)
     rp, col = gd.numpy()
-    P = atos.Graph(rp, col, gd.n, rank=rank, n_ranks=world, device=0, ctas_per_sm=1, watchdog_ms=120000,
+    P = atos.Graph(rp, col, gd.n, rank=rank, n_ranks=world, device=0, ctas_per_sm=1, watchdog_ms=600000,
                    channel_packets=64)
     adist.connect_graph(P, world)
     dist.barrier()

@@ -58,7 +58,7 @@ def test_struct_layouts_match_header():
 
 
 def test_version():
-    assert atos.load().atos_version() == 3
+    assert atos.load().atos_version() == 4
 
 
 def test_partition_balanced_matches_definition():

@@ -168,6 +168,24 @@ def test_bad_arguments():
 
 
 @pytest.mark.slow
+@pytest.mark.parametrize("vr", [2, 4, 8])
+def test_rmat24_config2_full_size_virtual_ranks(vr):
+    """configs[2] at full size with the multi-rank protocol (2/4/8 ranks, virtual on
+    this one GPU): depths and min-id parents bit-exact vs the oracle, aggregation
+    on and off (identical depth arrays for p in {1,2,4,8})."""
+    g = inputs.make_config("rmat24", device="cuda")
+    src = inputs.bfs_sources(g, 3)[vr.bit_length() - 2]
+    rpn, coln = g.numpy()
+    want = oracle.bfs(rpn, coln, src)
+    pwant = oracle.bfs_parents_minid(rpn, coln, want, src)
+    for agg in (1, 0):
+        with atos.Graph(g.row_ptr, g.col, g.n, virtual_ranks=vr, agg_enabled=agg) as G:
+            d, par = G.bfs(src, parent=True)
+        assert np.array_equal(d, want), (vr, agg)
+        assert np.array_equal(par, pwant), (vr, agg)
+
+
+@pytest.mark.slow
 def test_rmat24_config2_full_size():
     """BASELINE configs[2] at full size, the launch configuration bench.py times."""
     g = inputs.make_config("rmat24", device="cuda")

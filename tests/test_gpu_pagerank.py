@@ -185,3 +185,31 @@ def test_rmat26_8ranks_config4_invariant_full_size():
         rhs.index_add_(0, g.col[a:a + step].to(torch.int64), ALPHA * share[row[a:a + step]])
     lhs = r_out + s_out
     assert float((lhs - rhs).abs().max()) <= 1e-9 * max(1.0, float(lhs.abs().max()))
+
+
+@pytest.mark.slow
+def test_rmat26_8ranks_config4_vs_oracle_full_size():
+    """BASELINE configs[4] at full size in bench.py's launch configuration (8 ranks,
+    virtual on one GPU; aggregation on and off) compared element by element with
+    the oracle's Jacobi PageRank (OpenMP, 1e-12): max <= 1e-6, L1 <= 1e-5 after
+    normalisation, every residual in [0, eps)."""
+    import torch
+    g = inputs.make_config("rmat26_pr", device="cuda")
+    n = g.n
+    r_out = torch.empty(n, dtype=torch.float64, device="cuda")
+    s_out = torch.empty(n, dtype=torch.float64, device="cuda")
+    got = []
+    for agg in (1, 0):
+        with atos.Graph(g.row_ptr, g.col, n, relabel=0, virtual_ranks=8, agg_enabled=agg) as P:
+            P.pagerank(ALPHA, EPS, rank_out=r_out, residual_out=s_out)
+            P.sync()
+        assert bool((s_out >= 0).all()) and bool((s_out < EPS).all())
+        got.append((r_out / r_out.sum()).cpu().numpy())
+    rp, col = g.numpy()
+    del g
+    torch.cuda.empty_cache()
+    p, it, delta = oracle.pagerank(rp, col, ALPHA, 1e-12)
+    assert delta <= 1e-12
+    for p_hat in got:
+        err = np.abs(p_hat - p)
+        assert err.max() <= 1e-6 and err.sum() <= 1e-5, (err.max(), err.sum())
