@@ -23,6 +23,11 @@
 
 using namespace atos;
 
+constexpr int kColPad = 4;   // column arrays end with 4 spare entries (16-B loads of a row's last edges)
+constexpr int64_t kHubAutoN = 1 << 21;   // hub bounds cover the top 2^21 ids by default (16 KB of shared memory)
+constexpr int64_t kHubMaxN = 1 << 22;
+
+
 // ---------------------------------------------------------------------------
 // errors
 // ---------------------------------------------------------------------------
@@ -126,8 +131,8 @@ static bool valid_cfg(const atos_config &c) {
            c.watchdog_ms >= 0 && c.n_ranks >= 1 && c.n_ranks <= ATOS_MAX_RANKS && c.rank >= 0 &&
            c.rank < c.n_ranks && c.virtual_ranks >= 1 && c.virtual_ranks <= ATOS_MAX_RANKS &&
            !(c.virtual_ranks > 1 && c.n_ranks > 1) && c.ctas_per_sm >= 0 && c.device >= 0 &&
-           c.relabel >= 0 && c.relabel <= 2 && c.hub_cache >= -1 && c.hub_cache <= kHubMax &&
-           (c.hub_cache <= 0 || c.hub_cache % (32 * std::max(c.n_ranks, c.virtual_ranks)) == 0) &&
+           c.relabel >= 0 && c.relabel <= 2 && c.hub_cache >= -1 && c.hub_cache <= kHubMaxN &&
+           (c.hub_cache <= 0 || c.hub_cache % 128 == 0) &&
            (c.split_edges == 0 || c.split_edges == -1 ||
             (c.split_edges >= 256 && c.split_edges <= (1 << 20) && pow2(c.split_edges))) &&
            (c.pr_combine == 0 || c.pr_combine == 1) && (c.pool_retain == 0 || c.pool_retain == 1) &&
@@ -138,7 +143,7 @@ static bool valid_cfg(const atos_config &c) {
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, filt, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, ghost, total;
+    size_t ctrl, depth, filt, hcb, rank, res, ring, in_hdr, in_pay, free_m, staging, parent, ghost, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -155,6 +160,7 @@ struct Shape {
     int cp, pkt, stage_cap, ctas_per_rank, fetch;
     double ring_factor;
     int combine;       // PR ghost residuals allocated (n_ranks > 1 && pr_combine)
+    int hub_chunks;    // BFS hub bounds array (single rank)
 };
 
 static Layout make_layout(const Shape &S, const int64_t *part, int r) {
@@ -167,6 +173,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.ctrl = o;    o = al(o + sizeof(Ctrl));
     L.depth = o;   o = al(o + (size_t)S.n * 4);
     L.filt = o;    o = al(o + (size_t)S.n);
+    L.hcb = o;     o = al(o + (size_t)S.hub_chunks);
     L.rank = o;    o = al(o + (size_t)L.n_r * 8);
     L.res = o;     o = al(o + (size_t)L.n_r * 8);
     L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
@@ -225,7 +232,8 @@ struct atos_graph {
     int32_t *d_depth_full = nullptr;
     int32_t *d_perm = nullptr;     // degree relabeling: old -> new (NULL = identity)
     int32_t *d_inv = nullptr;      //                    new -> old
-    int hc_per_rank = 0;           // BFS hub-cache entries per rank block
+    int hub_n = 0;                 // BFS hub bounds: ids [0, hub_n) covered (single rank, relabeled graphs)
+    int hub_chunks = 0;            // hub_n / 128 rounded up to a multiple of 16 (array size)
     bool skewed = true;            // max degree >= 32 x mean degree (set when an auto option needs it)
     int64_t **d_accs = nullptr;
     uint64_t epoch = 0;
@@ -285,8 +293,8 @@ static void dfree(const atos_graph *g, void *p) {
 }
 
 // dynamic shared memory of the worker: Smem, plus the BFS hub cache (one nibble per entry)
-static size_t worker_smem(int app, int hc_entries) {
-    return sizeof(Smem) + (app == kApBfs ? (size_t)hc_entries / 2 : 0);
+static size_t worker_smem(int app, int hub_chunks) {
+    return sizeof(Smem) + (app == kApBfs ? (size_t)hub_chunks : 0);
 }
 
 // Dynamic smem limit, then the smallest shared-memory carve-out that still holds
@@ -324,6 +332,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     const Layout &L = me.L;
     d.depth = (uint32_t *)(b + L.depth);
     d.filt = (uint8_t *)(b + L.filt);
+    d.hcb = (uint8_t *)(b + L.hcb);
     d.pr_rank = (double *)(b + L.rank);
     d.pr_res = (double *)(b + L.res);
     d.pr_q = pr_q_of(L.n_r);
@@ -469,6 +478,14 @@ static atos_status upload_views(atos_graph *g) {
 
 static KParams make_params(atos_graph *g);
 
+// hub bounds: vertices covered (multiple of 128, <= n) and the array size
+static int hub_n_for(const atos_config &cfg, int64_t n) {
+    int64_t h = cfg.hub_cache < 0 ? kHubAutoN : cfg.hub_cache;
+    h = std::min<int64_t>(h, n);
+    return (int)(h - h % 128);
+}
+static int hub_chunks_for(int hub_n) { return ((hub_n / 128 + 15) / 16) * 16; }
+
 extern "C" atos_status atos_graph_free(atos_graph *g) {
     if (!g) return ATOS_OK;
     cudaSetDevice(g->cfg.device);
@@ -527,7 +544,7 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
     else atos_partition_balanced(n, n_ranks, pt.data());
     Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs),
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
-            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine};
+            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0};
     *bytes_out = make_layout(S, pt.data(), rank).total;
     return ATOS_OK;
 }
@@ -600,7 +617,7 @@ static atos_status relabel_rows(atos_graph *g, LocalRank &me) {
     int32_t *col_new = nullptr;
     CU(dmalloc(g, &deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
     CU(dmalloc(g, &rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
-    CU(dmalloc(g, &col_new, (size_t)std::max<int64_t>(me.m_r, 1) * 4)); fr.p.push_back(col_new);
+    CU(dmalloc(g, &col_new, ((size_t)me.m_r + kColPad) * 4)); fr.p.push_back(col_new);
     new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
     size_t tb = 0;
     CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
@@ -635,7 +652,7 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
     int32_t *col_new = nullptr;
     CU(dmalloc(g, &deg, (size_t)(nr + 1) * 8)); fr.p.push_back(deg);
     CU(dmalloc(g, &rp_new, (size_t)(nr + 1) * 8)); fr.p.push_back(rp_new);
-    CU(dmalloc(g, &col_new, (size_t)std::max<int64_t>(m, 1) * 4)); fr.p.push_back(col_new);
+    CU(dmalloc(g, &col_new, ((size_t)m + kColPad) * 4)); fr.p.push_back(col_new);
     new_degrees_kernel<<<1024, 256, 0, st>>>(me.row_ptr, g->d_inv, v0, nr, deg);
     size_t tb = 0;
     CU(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, rp_new, (int64_t)(nr + 1), st));
@@ -762,15 +779,11 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     // (the persisting carve-out itself is sized per launch to the window, see launch_worker:
     //  a carve-out larger than the window would only shrink the L2 left to everything else)
     if (!prop.cooperativeLaunch) return fail(ATOS_ERR_CUDA, "device lacks cooperative launch");
-    // hub cache: entries per rank block (needed for the BFS kernel's shared memory)
-    {
-        int hc = cfg.hub_cache;
-        if (hc < 0) hc = 0;   // auto = off: measured slower than the L1 on RMAT-24/26
-        hc -= hc % (32 * g->p);
-        g->hc_per_rank = hc / g->p;
-    }
+    // hub bounds (atos_bfs1.cuh): the largest size they can take decides the BFS
+    // kernel's shared memory; the actual size is set once relabeling is known
+    const int hub_max = g->p == 1 ? hub_n_for(cfg, n) : 0;
     const int want = cfg.ctas_per_sm > 0 ? cfg.ctas_per_sm : 1024 / kThreads;
-    const size_t smem_bfs = worker_smem(kApBfs, g->hc_per_rank * g->p), smem_pr = worker_smem(kApPr, 0);
+    const size_t smem_bfs = worker_smem(kApBfs, hub_chunks_for(hub_max)), smem_pr = worker_smem(kApPr, 0);
     int occ0 = 0, occ1 = 0, occ2 = 0, occ3 = 0;   // single- and multi-rank specialisations
     CU((kernel_setup<kApBfs, false>(occ0, smem_bfs, want)));
     CU((kernel_setup<kApPr, false>(occ1, smem_pr, want)));
@@ -790,7 +803,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
     g->grid = cpr * g->n_local;
     g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs), cpr,
-                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine};
+                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0};
 
     if (cfg.stream) {
         g->stream = (cudaStream_t)cfg.stream;
@@ -811,6 +824,12 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         if (rs != ATOS_OK) return rs;
     }
 
+    // hub bounds only on relabeled (skewed) single-rank graphs: ids [0, hub_n) are the hubs
+    if (hub_max > 0 && g->d_perm) {
+        g->hub_n = hub_max;
+        g->hub_chunks = hub_chunks_for(hub_max);
+        g->S.hub_chunks = g->hub_chunks;
+    }
     unsigned long long *d_bad = nullptr;
     CU(cudaMalloc(&d_bad, sizeof(unsigned long long)));
     CU(cudaMemsetAsync(d_bad, 0, sizeof(unsigned long long), g->stream));
@@ -830,7 +849,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         const char *se = std::getenv("ATOS_LOAD_STREAMED");
         const bool streamed = g->d_perm && me.m_r > 0 && !rp_dev && !is_device_ptr(col) && !(se && se[0] == '0');
         CU(dmalloc(g, &me.row_ptr, (size_t)(nr + 1) * 8));
-        if (!streamed) CU(dmalloc(g, &me.col, (size_t)std::max<int64_t>(me.m_r, 1) * 4));
+        if (!streamed) CU(dmalloc(g, &me.col, ((size_t)me.m_r + kColPad) * 4));
         CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
         if (me.m_r > 0 && !streamed)
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
@@ -943,7 +962,12 @@ static KParams make_params(atos_graph *g) {
     kp.filter = g->cfg.probe_filter == 1 ||
                 (g->cfg.probe_filter == 2 && (g->skewed ||
                                               (size_t)g->n * 4 > (g->persist_max ? g->persist_max : (size_t)64 << 20)));
-    kp.hc_per_rank = g->hc_per_rank;
+    kp.hub_n = g->hub_n;
+    kp.hub_chunks = g->hub_chunks;
+    // lean single-rank BFS expansion (atos_bfs1.cuh) for the default relaxation
+    // (filter + red.min); ATOS_BFS_V1 selects the generic expansion (A/B)
+    kp.bfs1 = g->p == 1 && kp.filter && kp.relax_red && !std::getenv("ATOS_BFS_V1");
+    if (!kp.bfs1) kp.hub_n = kp.hub_chunks = 0;
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
     kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
@@ -1032,7 +1056,7 @@ static atos_status build_discrete_graph(atos_graph *g, const KParams &kp) {
     wk.func = (void *)worker_discrete_kernel<APP>;
     wk.gridDim = dim3(g->grid);
     wk.blockDim = dim3(kThreads);
-    wk.sharedMemBytes = (unsigned)worker_smem(APP, kp.hc_per_rank * g->p);
+    wk.sharedMemBytes = (unsigned)worker_smem(APP, kp.hub_chunks);
     wk.kernelParams = w_args;
     CU(cudaGraphAddKernelNode(&wnode, body, nullptr, 0, &wk));
     cudaAccessPolicyWindow win{};
@@ -1060,7 +1084,7 @@ static atos_status launch_worker(atos_graph *g, KParams &kp) {
     cudaLaunchConfig_t lc{};
     lc.gridDim = dim3(g->grid);
     lc.blockDim = dim3(kThreads);
-    lc.dynamicSmemBytes = worker_smem(APP, kp.hc_per_rank * g->p);
+    lc.dynamicSmemBytes = worker_smem(APP, kp.hub_chunks);
     lc.stream = g->stream;
     cudaLaunchAttribute at[2];
     int na = 0;

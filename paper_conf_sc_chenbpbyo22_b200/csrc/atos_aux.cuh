@@ -37,6 +37,8 @@ __global__ void init_bfs_kernel(KParams kp) {
             R.depth[i] = kInf;
             R.filt[i] = 255;
         }
+        for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < kp.hub_chunks; i += (int64_t)gridDim.x * blockDim.x)
+            R.hcb[i] = 255;     // hub bounds: unknown
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
 }

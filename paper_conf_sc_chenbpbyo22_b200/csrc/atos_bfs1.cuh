@@ -1,0 +1,267 @@
+// atos_bfs1.cuh -- the single-rank BFS expansion of the persistent worker
+// (Listing 5's neighbour loop, re-planned for sm_100a).
+//
+// Included by atos_worker.cuh; used by worker_body for BFS with one rank, the
+// probe filter and fire-and-forget relaxation (the defaults on every graph).
+//
+// Two ideas, both aimed at the two limits ncu showed for the generic
+// expansion: issued instructions per edge and the L1TEX wavefront rate of the
+// per-edge random probe (one 128-B line per lane, ~1 per SM clock: 285 G
+// probes/s measured, profiles/r1/micro_denominators.json).
+//
+// 1. Degree classes inside a batch (the paper's thread / warp / CTA load
+//    balancing by degree).  Rows of >= kLong edges -- hub pieces
+//    and long rows -- are cut into 128-edge chunks aligned to 16 B: a warp's
+//    chunk belongs to ONE row, so the row record is read once per chunk
+//    (warp-uniform candidate depth) and every lane loads its 4 edges with one
+//    LDG.128.  Short rows share a packed edge space mapped by the per-batch edge
+//    map (one bitmap word + one row index per 32 edges) to a 16-B row record.
+//
+// 2. Hub bounds.  After degree relabeling ids
+//    [0, hub_n) are the graph's highest-degree vertices, which receive most edge
+//    endpoints of a skewed graph (top 2^21 of RMAT-22: 0.97 of all endpoints).
+//    Chunk c = ids [128c, 128c + 128) has a global byte hcb[c] holding an UPPER
+//    BOUND of the largest probe-filter value in the chunk: every scan of the
+//    filter gives one (filter values only decrease; racing plain stores of two
+//    scans leave one of two valid bounds), and the warps of all workers re-scan
+//    all chunks once per batch (hub_refresh).  Every worker copies the array into
+//    shared memory per batch (hub_copy).  An edge to a hub u with candidate
+//    depth nd where hcb[u / 128] <= nd provably cannot improve u (depth(u) <=
+//    filt(u) <= bound <= nd), so it is retired by one shared-memory byte load
+//    instead of a global probe.  Exactness is unchanged: only edges that
+//    cannot improve are skipped.
+#pragma once
+// (included inside namespace atos by atos_worker.cuh)
+
+__device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
+    int4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "l"(ptr), "l"(pol));
+    return v;
+}
+
+// Re-scan this warp's share of the hub chunks into the global bounds.
+__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta) {
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t C = (uint32_t)kp.hub_n >> 7;            // (the array's padding stays 255)
+    const uint32_t GW = (uint32_t)kp.ctas_per_rank * kWarps;
+    const uint32_t *f = reinterpret_cast<const uint32_t *>(s.R.filt);
+    for (uint32_t c = (uint32_t)cta * kWarps + w; c < C; c += GW) {
+        const uint32_t x = __ldcg(f + (size_t)c * 32 + lane);     // the chunk's 128 filter bytes, from L2
+        const uint32_t m = max(max(x & 255u, (x >> 8) & 255u), max((x >> 16) & 255u, x >> 24));
+        const uint32_t cm = __reduce_max_sync(kFull, m);
+        if (lane == 0) s.R.hcb[c] = (uint8_t)cm;
+    }
+}
+
+// Copy the global hub bounds into this worker's shared memory (hub_chunks is a
+// multiple of 16).  Callers order it with a block barrier before use.
+__device__ __forceinline__ void hub_copy(Smem &s, const KParams &kp) {
+    uint4 *dst = reinterpret_cast<uint4 *>(hub_base(s));
+    const uint4 *src = reinterpret_cast<const uint4 *>(s.R.hcb);
+    for (int i = threadIdx.x; i < kp.hub_chunks / 16; i += kThreads) dst[i] = __ldcg(src + i);
+}
+
+// Relax N edges per lane (u[k] < 0: no edge): hub-bound test, filter probe,
+// red.min + filter store on the probe's verdict (relax_red; duplicates are
+// skipped at pop by the pending bit, the flush fences before publishing).
+template <int N>
+__device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                           const uint32_t (&nd)[N], uint32_t &msk, uint32_t &hits) {
+    uint32_t *const depth = s.R.depth;
+    uint8_t *const filt = s.R.filt;
+    const uint32_t H = (uint32_t)kp.hub_n;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        if ((uint32_t)u[k] < H) {     // (u < 0 is huge unsigned: not a hub)
+            const uint32_t hb = hcs[(uint32_t)u[k] >> 7];
+            if (hb <= nd[k] && hb != 255u) {
+                u[k] = -1;
+                ++hits;
+            }
+        }
+    }
+    uint32_t f[N];
+#pragma unroll
+    for (int k = 0; k < N; ++k) f[k] = u[k] >= 0 ? ldg_u8(filt + u[k]) : 0u;
+    msk = 0;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        if (u[k] >= 0 && (nd[k] < f[k] || f[k] == 255u)) {
+            red_min_u32(depth + u[k], dw_make(nd[k]));
+            stg_u8(filt + u[k], filt_of(nd[k]));
+            msk |= 1u << k;
+        }
+    }
+}
+
+// largest li in [0, NL) with lq0[li] <= c (lq0[0] == 0 <= c)
+__device__ __forceinline__ uint32_t long_row_of(const BatchBuf &bb, uint32_t NL, uint32_t c) {
+    uint32_t lo = 0, hi = NL - 1;
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (bb.lq0[mid] <= c) lo = mid; else hi = mid - 1;
+    }
+    return lo;
+}
+
+__device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t NL, uint32_t NLC, uint32_t ES,
+                            uint32_t &wn) {
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int32_t *const col = s.R.col;
+    const uint8_t *const hcs = hub_base(s);
+    const uint64_t pol = policy_evict_first();
+    const uint32_t below = lane == 31 ? 0xFFFFFFFEu : (((2u << lane) - 1u) & ~1u);
+    const uint32_t ntot = NLC + (ES + kLong - 1) / kLong;
+    const int64_t vb = s.R.v_begin;
+    uint32_t hits = 0;
+    for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
+        int32_t u[4];
+        uint32_t nd[4];
+        if (c < NLC) {
+            // long row chunk: one row, 16-B aligned, 4 edges per lane in one LDG.128
+            const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_of(bb, NL, c);
+            const BRec r = bb.rec[kThreads - 1 - li];
+            const uint32_t lo = (uint32_t)(r.base & 3);
+            const int64_t a = r.base - lo;
+            const uint32_t rel = (c - bb.lq0[li]) * (uint32_t)kLong + 4u * lane;   // edge offset from a
+            const uint32_t end = lo + r.len;
+            int4 v = make_int4(-1, -1, -1, -1);
+            if (rel < end) v = ld_stream4(col + a + rel, pol);   // may read <= 3 entries past the row (padded array)
+            u[0] = (rel >= lo && rel < end) ? v.x : -1;
+            u[1] = (rel + 1 >= lo && rel + 1 < end) ? v.y : -1;
+            u[2] = (rel + 2 >= lo && rel + 2 < end) ? v.z : -1;
+            u[3] = (rel + 3 < end) ? v.w : -1;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) nd[k] = r.nd;
+        } else {
+            // short rows: packed edge space, coalesced 4-B column loads
+            const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const uint32_t e = c0 + 32u * k + lane;
+                u[k] = -1;
+                nd[k] = 0;
+                if (e < ES) {
+                    const uint32_t wd = e >> 5;
+                    const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
+                    u[k] = ld_stream(col + r.base + e, pol);
+                    nd[k] = r.nd;
+                }
+            }
+        }
+        uint32_t msk;
+        relax_bfs1<4>(s, kp, hcs, u, nd, msk, hits);
+        if (__any_sync(kFull, msk != 0)) {
+            uint32_t item[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(u[k] - vb);
+            warp_append_mask<4>(s, w, wn, msk, item, true);
+        }
+    }
+    if (kp.hub_n) {
+        hits = __reduce_add_sync(kFull, hits);
+        if (lane == 0 && hits) atomicAdd(&s.c_hub, (unsigned long long)hits);
+    }
+}
+
+// Load per-vertex info of the batch s.v[0..B), classify rows, build the maps,
+// refresh + copy the hub bounds, expand.  (Single rank, filter + relax_red.)
+__device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
+    const RankDev &R = s.R;
+    BatchBuf &bb = s.bb[0];
+    const int tid = threadIdx.x;
+    int64_t deg = 0, b = 0;
+    uint32_t npc = 0, nd = 0;
+    if (tid < B) {
+        const uint32_t it = bb.v[tid];
+        if (it & kPieceBit) {
+            // a piece of a split row: edges [piece * split, (piece+1) * split) of v,
+            // relaxed with v's current depth (a valid bound: depths only decrease,
+            // and a newer depth re-expands the whole row anyway)
+            const uint32_t v = it & 0xFFFFu, pc = (it >> 16) & 0x7FFFu;
+            const int64_t rb = ldg_i64_nc(R.row_ptr + v), re = ldg_i64_nc(R.row_ptr + v + 1);
+            b = rb + (int64_t)pc * kp.split;
+            deg = re - b < (int64_t)kp.split ? re - b : (int64_t)kp.split;
+            const uint32_t d = dw_depth(ld_relaxed_gpu_u32(R.depth + R.v_begin + v));
+            nd = d + 1;
+            if (d == kDepthInf || deg < 0) deg = 0;
+        } else {
+            const uint32_t v = it;
+            b = ldg_i64_nc(R.row_ptr + v);
+            deg = ldg_i64_nc(R.row_ptr + v + 1) - b;
+            // claim the expansion of v at its current depth; stale duplicates see
+            // the pending bit already cleared and are skipped
+            const uint32_t old = atom_and_u32(R.depth + R.v_begin + v, ~1u);
+            const uint32_t d = dw_depth(old);
+            nd = d + 1;
+            if (!(old & 1u) || d == kDepthInf) deg = 0;
+            if (kp.split > 0 && deg > 2 * (int64_t)kp.split && (int64_t)v < kPieceVMax &&
+                deg <= (int64_t)kp.split * kPieceMax) {
+                npc = (uint32_t)((deg - 1) / kp.split);   // pieces 1..npc go to the ring
+                deg = kp.split;
+            }
+        }
+    }
+    if (kp.hub_chunks > 0) hub_refresh(s, kp, cta);       // overlaps the row loads above
+    if (kp.split > 0 && __syncthreads_or(npc > 0)) {
+        // publish the pieces before expanding, so idle workers start on them now;
+        // T grows before this batch's F, so termination cannot be declared early
+        int64_t pex;
+        const int64_t ptot = block_exscan(s, (int64_t)npc, pex);
+        if (tid == 0) {
+            s.b64[2] = atomicAdd((unsigned long long *)&R.ctrl->tail.v, (unsigned long long)ptot);
+            s.c_pushes += (unsigned long long)ptot;
+        }
+        __syncthreads();
+        const uint64_t pbase = s.b64[2] + (uint64_t)pex;
+        for (uint32_t i = 0; i < npc; ++i)
+            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
+    }
+    if (kp.hub_chunks > 0) hub_copy(s, kp);               // ordered before use by the scan's barriers
+    for (int i = tid; i < kBitW; i += kThreads) bb.bm[i] = 0u;
+    // one scan for four counts: long chunks [40,64) | long rows [30,40) | short edges [10,30) | short rows [0,10)
+    const bool lng = deg >= kLong;
+    const uint32_t lo = (uint32_t)(b & 3);
+    const uint32_t nch = lng ? (uint32_t)((deg + lo + kLong - 1) / kLong) : 0u;
+    const int64_t x = lng ? (((int64_t)nch << 40) | (1ll << 30)) : ((deg << 10) | (deg > 0 ? 1 : 0));
+    int64_t ex;
+    const int64_t tot = block_exscan(s, x, ex);
+    const uint32_t NLC = (uint32_t)(tot >> 40), NL = (uint32_t)((tot >> 30) & 1023), ES = (uint32_t)((tot >> 10) & 0xFFFFF);
+    if (deg > 0) {
+        if (lng) {
+            const uint32_t li = (uint32_t)((ex >> 30) & 1023), q0 = (uint32_t)(ex >> 40);
+            BRec r;
+            r.base = b;
+            r.nd = nd;
+            r.len = (uint32_t)deg;
+            bb.rec[kThreads - 1 - li] = r;
+            bb.lq0[li] = q0;
+            for (uint32_t q = q0; q < q0 + nch && q < (uint32_t)kLcv; ++q) bb.lcv[q] = (uint16_t)li;
+        } else {
+            const uint32_t off = (uint32_t)((ex >> 10) & 0xFFFFF), nz = (uint32_t)(ex & 1023);
+            BRec r;
+            r.base = b - (int64_t)off;
+            r.nd = nd;
+            r.len = 0;
+            bb.rec[nz] = r;
+            atomicOr(&bb.bm[off >> 5], 1u << (off & 31));
+            for (uint32_t wd = (off + 31) >> 5; wd <= ((off + (uint32_t)deg - 1) >> 5); ++wd) bb.rowmap[wd] = (uint16_t)nz;
+        }
+    }
+    // edges of the batch (statistics): per-warp sums, one smem atomic per warp
+    unsigned long long de = (unsigned long long)deg;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) de += __shfl_xor_sync(kFull, de, o);
+    if ((tid & 31) == 0 && de) atomicAdd(&s.c_edges, de);
+    __syncthreads();
+    if (NLC + ES > 0) {
+        const int w = tid >> 5;
+        uint32_t wn = s.wn[w];
+        expand_bfs1(s, bb, kp, NL, NLC, ES, wn);
+        __syncwarp();
+        if ((tid & 31) == 0) s.wn[w] = wn;
+    }
+}
+

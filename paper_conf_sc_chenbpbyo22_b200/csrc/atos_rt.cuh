@@ -251,6 +251,7 @@ struct RankDev {
     // application state (own memory)
     uint32_t *depth;             // BFS: [n] global-indexed words dw (owned + ghost filter)
     uint8_t *filt;               // BFS: [n] probe filter, an upper bound of depth saturated at 255
+    uint8_t *hcb;                // BFS hub bounds: [hub_chunks] upper bound of max filt over 128 hub ids
     double *pr_rank;             // PR: [n_r], stored at pr_slot(local id)
     double *pr_res;              // PR: [n_r], stored at pr_slot(local id)
     double *pr_ghost;            // PR combining: [n] unsent residual for remote vertices, at pr_slot(global id, pr_q_of(n)); NULL = off
@@ -297,7 +298,9 @@ struct KParams {
     int32_t relax_red;       // BFS: fire-and-forget red.min, enqueue on the probe's verdict
     int32_t pipe;            // BFS: software-pipelined expansion (two 128-edge chunks in flight)
     int32_t filter;          // BFS: probe the u8 filter instead of the depth words
-    int32_t hc_per_rank;     // BFS hub cache: entries per rank block (0 = off)
+    int32_t hub_n;           // BFS hub bounds: vertex ids [0, hub_n) covered (multiple of 2048; 0 = off)
+    int32_t hub_chunks;      // hub_n / 128
+    int32_t bfs1;            // single-rank BFS: the lean expansion of atos_bfs1.cuh (else the generic one)
     int32_t split;           // BFS row pieces: edges per piece (0 = off), see kPieceBit
     int32_t combine;         // PR sender-side residual combining (multi-rank)
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained

@@ -48,7 +48,6 @@ constexpr int kChunk = 32 * kU;      // edges per warp chunk
 constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr int kHubMax = 65536;       // max hub-cache entries per CTA (32 KB of nibbles; 2 CTAs/SM still fit)
 
 // BFS row pieces.  A popped row longer than
 // 2 x kp.split edges is cut: the popping worker expands the first kp.split edges
@@ -81,6 +80,15 @@ template <> struct AppTraits<kApPr> { static constexpr int kMsgBytes = 16; };
 constexpr int kBitW = 2048;
 constexpr int64_t kBitE = (int64_t)kBitW * 32;
 
+// One row of a popped batch in the single-rank BFS expansion (atos_bfs1.cuh).
+struct alignas(16) BRec {
+    int64_t base;    // short row: beg - (row's offset in the packed short edge space); long row: beg
+    uint32_t nd;     // candidate depth of the row's targets (popped depth + 1)
+    uint32_t len;    // long row: edges in the row (piece); short row: unused
+};
+constexpr int kLong = 128;           // rows of >= kLong edges are expanded as aligned 128-edge chunks
+constexpr int kLcv = 4096;           // long chunks whose row is precomputed per batch
+
 struct BatchBuf {
     uint32_t v[kThreads];          // local vertex ids
     uint64_t val[kThreads];        // depth (BFS) or delta bits (PR)
@@ -92,6 +100,12 @@ struct BatchBuf {
     uint32_t bm[kBitW];
     uint16_t rowmap[kBitW];
     uint16_t nzslot[kThreads];
+    // single-rank BFS expansion (atos_bfs1.cuh): one 16-B record per row -- short
+    // rows at [0, NZ) in edge-map order, long rows at [kThreads - NL, kThreads) --,
+    // the long-row chunk -> row map and the first chunk of every long row
+    BRec rec[kThreads];
+    uint16_t lcv[kLcv];
+    uint32_t lq0[kThreads];
 };
 
 // batch slot holding edge e (e = 32 * w + lane) from the edge map
@@ -101,7 +115,7 @@ __device__ __forceinline__ int bm_slot(const BatchBuf &bb, int64_t e, int lane) 
     return bb.nzslot[bb.rowmap[w] + __popc(bb.bm[w] & below)];
 }
 
-struct Smem {
+struct alignas(16) Smem {
     RankDev R;
     BatchBuf bb[1];
     uint32_t wout[kWarps][kWOut];  // per-warp local push staging
@@ -143,34 +157,8 @@ __device__ __forceinline__ int owner_of(const RankDev &R, int64_t u) {
     return r;
 }
 
-// ---------------------------------------------------------------------------
-// BFS hub cache.  After degree relabeling the first
-// hc_per_rank ids of every rank block are that block's highest-degree vertices,
-// which receive most of the edge endpoints of a skewed graph.  Every CTA keeps a
-// shared-memory nibble per such vertex holding an UPPER BOUND of its depth word
-// (15 = unknown / >= 15).  Depths only decrease, so any value ever observed (a
-// probe result, or nd after this CTA's own relaxation) stays an upper bound
-// forever; racy read-modify-writes of the shared byte can only lose an update,
-// which leaves an older, still valid bound.  hub <= nd proves that relaxing the
-// edge cannot improve the vertex, so the edge is retired without touching L2:
-// a shared-memory lookup replaces the random global probe, whose L1TEX cost
-// (one wavefront per distinct line) is the binding limit of the BFS expansion.
-// ---------------------------------------------------------------------------
+// Dynamic shared memory after Smem: the BFS hub bounds (atos_bfs1.cuh).
 __device__ __forceinline__ uint8_t *hub_base(Smem &s) { return reinterpret_cast<uint8_t *>(&s + 1); }
-
-__device__ __forceinline__ int hub_slot(const RankDev &R, int hpr, bool multi, int32_t u) {
-    if (!multi) return (uint32_t)u < (uint32_t)hpr ? u : -1;
-    const int o = owner_of(R, u);
-    const int64_t l = (int64_t)u - R.part[o];
-    return l < hpr ? o * hpr + (int)l : -1;
-}
-__device__ __forceinline__ uint32_t hub_get(const uint8_t *hc, int i) { return (hc[i >> 1] >> ((i & 1) * 4)) & 15u; }
-__device__ __forceinline__ void hub_put(uint8_t *hc, int i, uint32_t d) {
-    const uint32_t x = d < 15u ? d : 15u;
-    const int sh = (i & 1) * 4;
-    const uint32_t b = hc[i >> 1];
-    if (x < ((b >> sh) & 15u)) hc[i >> 1] = (uint8_t)((b & ~(15u << sh)) | (x << sh));
-}
 
 // Streaming loads of the column array: bypass L1, evict-first in L2 so that the
 // random-access state (depth / residual) stays L2-resident.
@@ -656,8 +644,8 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
 
 // ---------------------------------------------------------------------------
 // BFS relaxation of N edges per lane (u[k] = target or -1, nd[k] = candidate
-// depth): hub-cache lookup, probe (a stale word is larger, never smaller, so a
-// probe can only cause a redundant atomic), relaxation, hub-cache update.
+// depth): probe (a stale word is larger, never smaller, so a probe can only
+// cause a redundant atomic), then the relaxation.
 // Retired edges come back with u[k] = -1 and imp[k] = false.  Whole warp.
 // ---------------------------------------------------------------------------
 template <int N, bool MULTI>
@@ -667,24 +655,6 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
     uint32_t *const depth = R.depth;
     uint8_t *const filt = R.filt;
     const bool fl = kp.filter;
-    const int hpr = kp.hc_per_rank;
-    uint8_t *const hc = hub_base(s);
-    int hs[N];
-    if (hpr > 0) {
-        uint32_t hits = 0;
-#pragma unroll
-        for (int k = 0; k < N; ++k) {
-            hs[k] = u[k] >= 0 ? hub_slot(R, hpr, MULTI, u[k]) : -1;
-            const uint32_t hb = hs[k] >= 0 ? hub_get(hc, hs[k]) : 15u;
-            if (hb < 15u && hb <= nd[k]) {   // cannot improve: retired in shared memory (15 = unknown)
-                u[k] = -1;
-                hs[k] = -1;
-                ++hits;
-            }
-        }
-        const uint32_t tot = __reduce_add_sync(kFull, hits);
-        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(&s.c_hub, (unsigned long long)tot);
-    }
     uint32_t cur[N];
     if (fl) {
 #pragma unroll
@@ -720,16 +690,6 @@ __device__ __forceinline__ void bfs_relax(Smem &s, const KParams &kp, int32_t (&
             if (u[k] >= 0 && (fl ? filt_pass(cur[k], u[k], nd[k]) : ndw < cur[k])) {
                 imp[k] = atom_min_u32(depth + u[k], ndw) > ndw;
                 if (fl && imp[k]) filt_put(filt, u[k], nd[k], cur[k]);
-            }
-        }
-    }
-    if (hpr > 0) {
-        // after the relaxation depth(u) <= nd; a probe that made it unnecessary saw a smaller bound
-#pragma unroll
-        for (int k = 0; k < N; ++k) {
-            if (hs[k] >= 0) {
-                const uint32_t ob = fl ? filt_val(cur[k], u[k]) : dw_depth(cur[k]);
-                hub_put(hc, hs[k], ob < nd[k] ? ob : nd[k]);
             }
         }
     }
@@ -1024,8 +984,7 @@ __device__ void expand_warp_pipe(Smem &s, BatchBuf &bb, const KParams &kp, int c
 // BFS expansion, three-stage software pipeline (pipeline = 3): while chunk i
 // is relaxed (compare, red/atomicMin, append), the probes of chunk i+1 and the
 // column loads of chunk i+2 are already in flight, so a warp keeps two memory
-// round trips outstanding instead of waiting on col -> probe per chunk.  No hub
-// cache (the caller falls back to expand_warp when it is on).
+// round trips outstanding instead of waiting on col -> probe per chunk.
 // ---------------------------------------------------------------------------
 template <bool MULTI>
 __device__ __forceinline__ void probe_issue(const KParams &kp, const RankDev &R, const PipeStage &st,
@@ -1231,7 +1190,7 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         uint32_t wn = s.wn[w];
         // pipelined expansion pays off on low-degree (latency-bound, road-like) batches
 #ifdef ATOS_PIPE3   // experimental: raises register pressure (stack spills) of the default paths
-        if (APP == kApBfs && kp.pipe == 3 && kp.hc_per_rank == 0)
+        if (APP == kApBfs && kp.pipe == 3)
             expand_warp_pipe3<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         else
 #endif
@@ -1317,6 +1276,8 @@ __device__ void report_staged(Smem &s, const KParams &kp) {
     }
     __syncthreads();
 }
+
+#include "atos_bfs1.cuh"
 
 // ---------------------------------------------------------------------------
 // pop from the local ring: reserve-then-wait
@@ -1456,11 +1417,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         s.wn[tid] = 0;
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
-    if (APP == kApBfs && kp.hc_per_rank > 0) {   // hub cache: every bound unknown (15)
-        uint32_t *hc = reinterpret_cast<uint32_t *>(hub_base(s));   // (dynamic smem is only 8-B aligned)
-        const int n4 = kp.hc_per_rank * kp.ranks[lr].n_ranks / 8;
-        for (int i = tid; i < n4; i += kThreads) hc[i] = kFull;
-    }
+    if (APP == kApBfs && !MULTI && kp.hub_chunks > 0) hub_copy(s, kp);   // hub bounds: every chunk unknown (255)
     __syncthreads();
     constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
@@ -1505,7 +1462,12 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
 #ifdef ATOS_PROF
                     const long long pb1 = clock64();
 #endif
-                    process_batch<APP, MULTI>(s, kp, cta, B);
+                    if constexpr (APP == kApBfs && !MULTI) {
+                        if (kp.bfs1) process_batch_bfs1(s, kp, cta, B);
+                        else process_batch<APP, MULTI>(s, kp, cta, B);
+                    } else {
+                        process_batch<APP, MULTI>(s, kp, cta, B);
+                    }
 #ifdef ATOS_PROF
                     const long long pb2 = clock64();
                     if (tid == 0) s.prof[8] += (unsigned long long)(pb2 - pb1);

@@ -202,14 +202,16 @@ def test_rmat24_config2_full_size():
 @pytest.mark.parametrize("opts", [dict(relabel=0), dict(relabel=1, hub_cache=0), dict(relabel=1),
                                   dict(relabel=0, hub_cache=1024), dict(relabel=1, relax_red=0),
                                   dict(relabel=1, probe_filter=1), dict(relabel=1, pipeline=1),
-                                  dict(relabel=1, pipeline=0, hub_cache=32),
+                                  dict(relabel=1, pipeline=0, hub_cache=128),
+                                  dict(relabel=1, hub_cache=128 * 3), dict(relabel=1, hub_cache=1 << 22),
                                   dict(relabel=1, virtual_ranks=4, hub_cache=128),
                                   dict(relabel=1, virtual_ranks=3, hub_cache=96 * 64),
                                   dict(relabel=1, virtual_ranks=8, agg_enabled=0)])
 def test_relabel_and_hub_cache_same_depths_and_parents(opts):
-    """Degree relabeling and the shared-memory hub cache change the
-    internal order and retire edges without a probe; depths and the min-id
-    parents in the caller's ids must be unchanged."""
+    """Degree relabeling and the hub bounds (atos_bfs1.cuh: per-128-hub chunk
+    upper bounds in shared memory) change the internal order and retire edges
+    without a probe; depths and the min-id parents in the caller's ids must be
+    unchanged."""
     g = inputs.rmat(15, 16, 4, symmetric=True)
     rp, col = g.numpy()
     for s in inputs.bfs_sources(g, 2, seed=7):
@@ -225,7 +227,9 @@ def test_relabel_and_hub_cache_same_depths_and_parents(opts):
 
 
 def test_hub_cache_active_on_skewed_graph():
-    g = inputs.rmat(16, 16, 1, symmetric=True)
+    """On a skewed graph most edges point at hubs whose chunk bound is already
+    small: the hub bounds retire a large share of the edges without a probe."""
+    g = inputs.rmat(18, 16, 1, symmetric=True)
     rp, col = g.numpy()
     src = inputs.bfs_sources(g, 1)[0]
     with atos.Graph(rp, col, relabel=1, hub_cache=65536) as G:
@@ -369,3 +373,24 @@ def test_grid4900_config3_full_size():
     with atos.Graph(g.row_ptr, g.col, g.n) as G:
         for s in (0, g.n // 2 + 2450):
             assert np.array_equal(G.bfs(s), oracle.bfs(rpn, coln, s))
+
+
+@pytest.mark.parametrize("opts", [dict(), dict(split_edges=0), dict(split_edges=256), dict(hub_cache=0),
+                                  dict(fetch_size=3), dict(keep_items=64, keep_mode=1)])
+def test_bfs1_long_rows_alignment_and_chunk_map(opts):
+    """The single-rank expansion (atos_bfs1.cuh): rows of >= 128 edges start at every
+    alignment mod 4 and end ragged; a row of 700 000 edges without splitting has more
+    128-edge chunks than the per-batch chunk map (4096) and takes the search path;
+    the last row of the column array is long (16-B loads past its end read the
+    array's padding)."""
+    rng = np.random.default_rng(5)
+    n = 800000
+    edges = [(0, v) for v in range(1, 700001)]                       # one huge row (unsplittable with split 0)
+    for u in range(1, 3000):                                          # long rows of every length mod 4
+        d = 128 + int(rng.integers(0, 400))
+        edges += [(u, int(x)) for x in rng.integers(1, n, d)]
+    edges += [(n - 1, int(x)) for x in rng.integers(0, n, 300)]       # long last row
+    edges += [(v, 0) for v in range(1, 700001, 7)]                   # back edges to the hub
+    rp, col = csr_of(n, list(set(edges)))
+    for s in (0, 1, 17, n - 1):
+        run_and_check(rp, col, s, **opts)
