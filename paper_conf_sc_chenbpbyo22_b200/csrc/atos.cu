@@ -891,6 +891,14 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     CU(dmalloc(g, &g->d_depth_full, (size_t)n * 4));
     CU(cudaMalloc(&g->d_accs, sizeof(int64_t *) * kMaxRanks));
     g->connected = !g->multiproc;
+    for (int lr = 0; lr < g->n_local; ++lr)    // the 16-B column loads of atos_bfs1.cuh need this
+        if (((uintptr_t)g->loc[lr].col & 15) != 0)
+            return fail(ATOS_ERR_CUDA, "column array not 16-B aligned (%p)", (void *)g->loc[lr].col);
+    if (std::getenv("ATOS_DEBUG_PTRS"))
+        for (int lr = 0; lr < g->n_local; ++lr)
+            fprintf(stderr, "[atos] rank %d col %p row_ptr %p arena %p m_r %lld hub_n %d chunks %d smem %zu\n", lr,
+                    (void *)g->loc[lr].col, (void *)g->loc[lr].row_ptr, (void *)g->loc[lr].arena,
+                    (long long)g->loc[lr].m_r, g->hub_n, g->hub_chunks, worker_smem(kApBfs, g->hub_chunks));
     atos_status st = upload_views(g);
     if (st != ATOS_OK) return st;
     tr.mark(g->stream, "finish");

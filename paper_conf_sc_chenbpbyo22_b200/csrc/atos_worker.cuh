@@ -1417,8 +1417,8 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         s.wn[tid] = 0;
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
-    if (APP == kApBfs && !MULTI && kp.hub_chunks > 0) hub_copy(s, kp);   // hub bounds: every chunk unknown (255)
     __syncthreads();
+    // (hub bounds: the first process_batch_bfs1 copies them to shared memory before any use)
     constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
     if (tid == 0 && cta == 0) st_release_peer(kp.sys, &s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
