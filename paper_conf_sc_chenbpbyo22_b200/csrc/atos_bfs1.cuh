@@ -24,8 +24,8 @@
 //    BOUND of the largest probe-filter value in the chunk: every scan of the
 //    filter gives one (filter values only decrease; racing plain stores of two
 //    scans leave one of two valid bounds), and the warps of all workers re-scan
-//    all chunks once per batch (hub_refresh).  Every worker copies the array into
-//    shared memory per batch (hub_copy).  An edge to a hub u with candidate
+//    all chunks every few batches (hub_refresh).  Every worker copies the array
+//    into shared memory per batch with one TMA bulk copy (hub_copy_issue).  An edge to a hub u with candidate
 //    depth nd where hcb[u / 128] <= nd provably cannot improve u (depth(u) <=
 //    filt(u) <= bound <= nd), so it is retired by one shared-memory byte load
 //    instead of a global probe.  Exactness is unchanged: only edges that
@@ -41,26 +41,54 @@ __device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
     return v;
 }
 
-// Re-scan this warp's share of the hub chunks into the global bounds.
-__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta) {
+// Re-scan ONE hub chunk per warp per batch into the global bounds: batch r of a
+// worker's warp gw scans chunk gw + GW * (r mod ceil(C / GW)), so all chunks are
+// re-scanned every ceil(C / GW) batches of every worker (4 at RMAT-24/26 with
+// 2^21 hubs and 296 workers).  Called after the warp's expansion, where it
+// waits for the batch-end barrier anyway.
+__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta, uint32_t rnd) {
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t C = (uint32_t)kp.hub_n >> 7;            // (the array's padding stays 255)
     const uint32_t GW = (uint32_t)kp.ctas_per_rank * kWarps;
-    const uint32_t *f = reinterpret_cast<const uint32_t *>(s.R.filt);
-    for (uint32_t c = (uint32_t)cta * kWarps + w; c < C; c += GW) {
-        const uint32_t x = __ldcg(f + (size_t)c * 32 + lane);     // the chunk's 128 filter bytes, from L2
-        const uint32_t m = max(max(x & 255u, (x >> 8) & 255u), max((x >> 16) & 255u, x >> 24));
-        const uint32_t cm = __reduce_max_sync(kFull, m);
-        if (lane == 0) s.R.hcb[c] = (uint8_t)cm;
+    const uint32_t R = (C + GW - 1) / GW;
+    const uint32_t c = (uint32_t)cta * kWarps + w + GW * (rnd % R);
+    if (c >= C) return;
+    const uint32_t x = __ldcg(reinterpret_cast<const uint32_t *>(s.R.filt) + (size_t)c * 32 + lane);   // 128 B, from L2
+    const uint32_t m = max(max(x & 255u, (x >> 8) & 255u), max((x >> 16) & 255u, x >> 24));
+    const uint32_t cm = __reduce_max_sync(kFull, m);
+    if (lane == 0) s.R.hcb[c] = (uint8_t)cm;
+}
+
+// Copy the global hub bounds into this worker's shared memory with one TMA bulk
+// copy (cp.async.bulk, completion on an mbarrier), issued by one thread at the
+// start of the batch setup and waited for just before the expansion, so it
+// overlaps the row loads and the scans.  hub_chunks is a multiple of 16.
+__device__ __forceinline__ uint32_t smem_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void hub_copy_issue(Smem &s, const KParams &kp) {
+    const uint32_t bytes = (uint32_t)kp.hub_chunks;
+    const uint32_t mb = smem_addr(&s.hub_mbar);
+    // the previous batch's (generic-proxy) reads of the bounds precede this async-proxy overwrite
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_addr(hub_base(s))), "l"(s.R.hcb), "r"(bytes), "r"(mb) : "memory");
+}
+
+__device__ __forceinline__ void hub_copy_wait(const Smem &s, uint32_t parity) {
+    const uint32_t mb = smem_addr(&s.hub_mbar);
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                     : "=r"(done) : "r"(mb), "r"(parity) : "memory");
     }
 }
 
-// Copy the global hub bounds into this worker's shared memory (hub_chunks is a
-// multiple of 16).  Callers order it with a block barrier before use.
-__device__ __forceinline__ void hub_copy(Smem &s, const KParams &kp) {
-    uint4 *dst = reinterpret_cast<uint4 *>(hub_base(s));
-    const uint4 *src = reinterpret_cast<const uint4 *>(s.R.hcb);
-    for (int i = threadIdx.x; i < kp.hub_chunks / 16; i += kThreads) dst[i] = __ldcg(src + i);
+__device__ __forceinline__ void hub_mbar_init(Smem &s) {   // one thread, before the loop's first barrier
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(&s.hub_mbar)) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    s.hub_par = 0;
+    s.hub_rnd = 0;
 }
 
 // Relax N edges per lane (u[k] < 0: no edge): hub-bound test, filter probe,
@@ -106,9 +134,56 @@ __device__ __forceinline__ uint32_t long_row_of(const BatchBuf &bb, uint32_t NL,
     return lo;
 }
 
+struct Chunk1 {
+    int32_t u[4];
+    uint32_t nd[4];
+};
+
+// Column loads of chunk c (long: one row, LDG.128; short: packed edge space).
+__device__ __forceinline__ void load_chunk1(const BatchBuf &bb, const int32_t *col, uint64_t pol, uint32_t NL,
+                                            uint32_t NLC, uint32_t ES, uint32_t c, uint32_t lane, uint32_t below,
+                                            Chunk1 &ch) {
+    if (c < NLC) {
+        // long row chunk: one row, 16-B aligned, 4 edges per lane in one LDG.128
+        const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_of(bb, NL, c);
+        const BRec r = bb.rec[kThreads - 1 - li];
+        const uint32_t lo = (uint32_t)(r.base & 3);
+        const int64_t a = r.base - lo;
+        const uint32_t rel = (c - bb.lq0[li]) * (uint32_t)kLong + 4u * lane;   // edge offset from a
+        const uint32_t end = lo + r.len;
+        int4 v = make_int4(-1, -1, -1, -1);
+        if (rel < end) v = ld_stream4(col + a + rel, pol);   // may read <= 3 entries past the row (padded array)
+        ch.u[0] = (rel >= lo && rel < end) ? v.x : -1;
+        ch.u[1] = (rel + 1 >= lo && rel + 1 < end) ? v.y : -1;
+        ch.u[2] = (rel + 2 >= lo && rel + 2 < end) ? v.z : -1;
+        ch.u[3] = (rel + 3 < end) ? v.w : -1;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) ch.nd[k] = r.nd;
+    } else {
+        // short rows: packed edge space, coalesced 4-B column loads
+        const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const uint32_t e = c0 + 32u * k + lane;
+            ch.u[k] = -1;
+            ch.nd[k] = 0;
+            if (e < ES) {
+                const uint32_t wd = e >> 5;
+                const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
+                ch.u[k] = ld_stream(col + r.base + e, pol);
+                ch.nd[k] = r.nd;
+            }
+        }
+    }
+}
+
+// Expand the batch: each warp takes chunks w, w + 16, ...; the columns of its
+// next chunk are in flight while the current one is probed and relaxed (two
+// chunks of memory-level parallelism per warp).
 __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t NL, uint32_t NLC, uint32_t ES,
                             uint32_t &wn) {
-    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    const uint32_t lane = threadIdx.x & 31;
     const int32_t *const col = s.R.col;
     const uint8_t *const hcs = hub_base(s);
     const uint64_t pol = policy_evict_first();
@@ -116,49 +191,23 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
     const uint32_t ntot = NLC + (ES + kLong - 1) / kLong;
     const int64_t vb = s.R.v_begin;
     uint32_t hits = 0;
-    for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
-        int32_t u[4];
-        uint32_t nd[4];
-        if (c < NLC) {
-            // long row chunk: one row, 16-B aligned, 4 edges per lane in one LDG.128
-            const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_of(bb, NL, c);
-            const BRec r = bb.rec[kThreads - 1 - li];
-            const uint32_t lo = (uint32_t)(r.base & 3);
-            const int64_t a = r.base - lo;
-            const uint32_t rel = (c - bb.lq0[li]) * (uint32_t)kLong + 4u * lane;   // edge offset from a
-            const uint32_t end = lo + r.len;
-            int4 v = make_int4(-1, -1, -1, -1);
-            if (rel < end) v = ld_stream4(col + a + rel, pol);   // may read <= 3 entries past the row (padded array)
-            u[0] = (rel >= lo && rel < end) ? v.x : -1;
-            u[1] = (rel + 1 >= lo && rel + 1 < end) ? v.y : -1;
-            u[2] = (rel + 2 >= lo && rel + 2 < end) ? v.z : -1;
-            u[3] = (rel + 3 < end) ? v.w : -1;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) nd[k] = r.nd;
-        } else {
-            // short rows: packed edge space, coalesced 4-B column loads
-            const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-                const uint32_t e = c0 + 32u * k + lane;
-                u[k] = -1;
-                nd[k] = 0;
-                if (e < ES) {
-                    const uint32_t wd = e >> 5;
-                    const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
-                    u[k] = ld_stream(col + r.base + e, pol);
-                    nd[k] = r.nd;
-                }
-            }
-        }
+    uint32_t c = (uint32_t)w;
+    Chunk1 a;
+    if (c < ntot) load_chunk1(bb, col, pol, NL, NLC, ES, c, lane, below, a);
+    while (c < ntot) {
+        const uint32_t cn = c + kWarps;
+        Chunk1 b;
+        if (cn < ntot) load_chunk1(bb, col, pol, NL, NLC, ES, cn, lane, below, b);
         uint32_t msk;
-        relax_bfs1<4>(s, kp, hcs, u, nd, msk, hits);
+        relax_bfs1<4>(s, kp, hcs, a.u, a.nd, msk, hits);
         if (__any_sync(kFull, msk != 0)) {
             uint32_t item[4];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(u[k] - vb);
+            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(a.u[k] - vb);
             warp_append_mask<4>(s, w, wn, msk, item, true);
         }
+        a = b;
+        c = cn;
     }
     if (kp.hub_n) {
         hits = __reduce_add_sync(kFull, hits);
@@ -172,6 +221,12 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     const RankDev &R = s.R;
     BatchBuf &bb = s.bb[0];
     const int tid = threadIdx.x;
+    const bool hub = kp.hub_chunks > 0;
+    if (hub && tid == 0) {
+        s.hub_par ^= 1u;              // parity of this batch's copy (read by all threads after the scan's barriers)
+        s.hub_rnd++;
+        hub_copy_issue(s, kp);
+    }
     int64_t deg = 0, b = 0;
     uint32_t npc = 0, nd = 0;
     if (tid < B) {
@@ -204,7 +259,6 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
             }
         }
     }
-    if (kp.hub_chunks > 0) hub_refresh(s, kp, cta);       // overlaps the row loads above
     if (kp.split > 0 && __syncthreads_or(npc > 0)) {
         // publish the pieces before expanding, so idle workers start on them now;
         // T grows before this batch's F, so termination cannot be declared early
@@ -219,7 +273,6 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
         for (uint32_t i = 0; i < npc; ++i)
             ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
     }
-    if (kp.hub_chunks > 0) hub_copy(s, kp);               // ordered before use by the scan's barriers
     for (int i = tid; i < kBitW; i += kThreads) bb.bm[i] = 0u;
     // one scan for four counts: long chunks [40,64) | long rows [30,40) | short edges [10,30) | short rows [0,10)
     const bool lng = deg >= kLong;
@@ -255,6 +308,7 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) de += __shfl_xor_sync(kFull, de, o);
     if ((tid & 31) == 0 && de) atomicAdd(&s.c_edges, de);
+    if (hub) hub_copy_wait(s, s.hub_par ^ 1u);             // this batch's bounds have landed
     __syncthreads();
     if (NLC + ES > 0) {
         const int w = tid >> 5;
@@ -263,5 +317,6 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
+    if (hub) hub_refresh(s, kp, cta, s.hub_rnd);
 }
 

@@ -136,6 +136,9 @@ struct alignas(16) Smem {
     int32_t wave_valid;
     // CTA-cooperative inbound claim (cta_inbound)
     int32_t in_got, in_src, in_r;
+    // BFS hub bounds (atos_bfs1.cuh): TMA-copy completion barrier, its parity, batch counter
+    alignas(8) uint64_t hub_mbar;
+    uint32_t hub_par, hub_rnd;
     uint64_t in_cc;
     uint32_t in_off[33];
     unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
@@ -1417,8 +1420,8 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         s.wn[tid] = 0;
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
+    if (APP == kApBfs && !MULTI && tid == 0) hub_mbar_init(s);   // hub bounds: TMA completion barrier
     __syncthreads();
-    // (hub bounds: the first process_batch_bfs1 copies them to shared memory before any use)
     constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
     if (tid == 0 && cta == 0) st_release_peer(kp.sys, &s.R.peer_ctrl[0]->started[s.R.rank].v, kp.epoch);
