@@ -41,22 +41,31 @@ __device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
     return v;
 }
 
-// Re-scan ONE hub chunk per warp per batch into the global bounds: batch r of a
-// worker's warp gw scans chunk gw + GW * (r mod ceil(C / GW)), so all chunks are
-// re-scanned every ceil(C / GW) batches of every worker (4 at RMAT-24/26 with
-// 2^21 hubs and 296 workers).  Called after the warp's expansion, where it
-// waits for the batch-end barrier anyway.
-__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta, uint32_t rnd) {
+// Re-scan this warp's hub chunks into the global bounds, all chunks of the
+// graph once per batch of every worker: warp gw scans chunks gw + GW * j (up to
+// 4 per warp with 2^21 hubs and 296 workers), loads first, then the reductions.
+// Called after the warp's expansion, where it waits for the batch-end barrier.
+__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta) {
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t C = (uint32_t)kp.hub_n >> 7;            // (the array's padding stays 255)
     const uint32_t GW = (uint32_t)kp.ctas_per_rank * kWarps;
-    const uint32_t R = (C + GW - 1) / GW;
-    const uint32_t c = (uint32_t)cta * kWarps + w + GW * (rnd % R);
-    if (c >= C) return;
-    const uint32_t x = __ldcg(reinterpret_cast<const uint32_t *>(s.R.filt) + (size_t)c * 32 + lane);   // 128 B, from L2
-    const uint32_t m = max(max(x & 255u, (x >> 8) & 255u), max((x >> 16) & 255u, x >> 24));
-    const uint32_t cm = __reduce_max_sync(kFull, m);
-    if (lane == 0) s.R.hcb[c] = (uint8_t)cm;
+    const uint32_t c0 = (uint32_t)cta * kWarps + w;
+    const uint32_t *f = reinterpret_cast<const uint32_t *>(s.R.filt);
+    for (uint32_t cb = c0; cb < C; cb += 4 * GW) {
+        uint32_t x[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint32_t c = cb + GW * j;
+            x[j] = c < C ? __ldcg(f + (size_t)c * 32 + lane) : 0u;   // 128 B per chunk, from L2
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint32_t c = cb + GW * j;
+            const uint32_t m = max(max(x[j] & 255u, (x[j] >> 8) & 255u), max((x[j] >> 16) & 255u, x[j] >> 24));
+            const uint32_t cm = __reduce_max_sync(kFull, m);
+            if (lane == 0 && c < C) s.R.hcb[c] = (uint8_t)cm;
+        }
+    }
 }
 
 // Copy the global hub bounds into this worker's shared memory with one TMA bulk
@@ -99,7 +108,7 @@ __device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, con
                                            const uint32_t (&nd)[N], uint32_t &msk, uint32_t &hits) {
     uint32_t *const depth = s.R.depth;
     uint8_t *const filt = s.R.filt;
-    const uint32_t H = (uint32_t)kp.hub_n;
+    const uint32_t H = (kp.hub_dbg & 4) ? 0u : (uint32_t)kp.hub_n;
 #pragma unroll
     for (int k = 0; k < N; ++k) {
         if ((uint32_t)u[k] < H) {     // (u < 0 is huge unsigned: not a hub)
@@ -134,52 +143,47 @@ __device__ __forceinline__ uint32_t long_row_of(const BatchBuf &bb, uint32_t NL,
     return lo;
 }
 
-struct Chunk1 {
-    int32_t u[4];
-    uint32_t nd[4];
-};
-
-// Column loads of chunk c (long: one row, LDG.128; short: packed edge space).
-__device__ __forceinline__ void load_chunk1(const BatchBuf &bb, const int32_t *col, uint64_t pol, uint32_t NL,
-                                            uint32_t NLC, uint32_t ES, uint32_t c, uint32_t lane, uint32_t below,
-                                            Chunk1 &ch) {
-    if (c < NLC) {
-        // long row chunk: one row, 16-B aligned, 4 edges per lane in one LDG.128
-        const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_of(bb, NL, c);
-        const BRec r = bb.rec[kThreads - 1 - li];
-        const uint32_t lo = (uint32_t)(r.base & 3);
-        const int64_t a = r.base - lo;
-        const uint32_t rel = (c - bb.lq0[li]) * (uint32_t)kLong + 4u * lane;   // edge offset from a
-        const uint32_t end = lo + r.len;
+// Expand the batch: each warp takes chunks w, w + 16, ...  A long-row chunk is
+// kLongG groups of 128 edges of ONE row: every lane loads kLongG x 4 edges with
+// kLongG independent LDG.128s, so a warp keeps kLongG x 512 B of the column
+// stream in flight (memory-level parallelism is what bounds the stream: a
+// warp's chunk is a dependent column -> probe -> relax chain).  A short chunk
+// is 128 edges of the packed short-row edge space.
+template <int G>
+__device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KParams &kp, const int32_t *col,
+                                           uint64_t pol, uint32_t NL, uint32_t c, uint32_t lane, const uint8_t *hcs,
+                                           int64_t vb, uint32_t &wn, uint32_t &hits) {
+    const int w = threadIdx.x >> 5;
+    const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_of(bb, NL, c);
+    const BRec r = bb.rec[kThreads - 1 - li];
+    const uint32_t lo = (uint32_t)(r.base & 3);
+    const int64_t a = r.base - lo;
+    const uint32_t rel0 = (c - bb.lq0[li]) * (uint32_t)(kLong * G) + 4u * lane;   // edge offset from a
+    const uint32_t end = lo + r.len;
+    int32_t u[4 * G];
+    uint32_t nd[4 * G];
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        const uint32_t rel = rel0 + (uint32_t)kLong * g;
         int4 v = make_int4(-1, -1, -1, -1);
         if (rel < end) v = ld_stream4(col + a + rel, pol);   // may read <= 3 entries past the row (padded array)
-        ch.u[0] = (rel >= lo && rel < end) ? v.x : -1;
-        ch.u[1] = (rel + 1 >= lo && rel + 1 < end) ? v.y : -1;
-        ch.u[2] = (rel + 2 >= lo && rel + 2 < end) ? v.z : -1;
-        ch.u[3] = (rel + 3 < end) ? v.w : -1;
+        u[4 * g + 0] = (rel >= lo && rel < end) ? v.x : -1;
+        u[4 * g + 1] = (rel + 1 >= lo && rel + 1 < end) ? v.y : -1;
+        u[4 * g + 2] = (rel + 2 >= lo && rel + 2 < end) ? v.z : -1;
+        u[4 * g + 3] = (rel + 3 < end) ? v.w : -1;
+    }
 #pragma unroll
-        for (int k = 0; k < 4; ++k) ch.nd[k] = r.nd;
-    } else {
-        // short rows: packed edge space, coalesced 4-B column loads
-        const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
+    for (int k = 0; k < 4 * G; ++k) nd[k] = r.nd;
+    uint32_t msk;
+    relax_bfs1<4 * G>(s, kp, hcs, u, nd, msk, hits);
+    if (__any_sync(kFull, msk != 0)) {
+        uint32_t item[4 * G];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-            const uint32_t e = c0 + 32u * k + lane;
-            ch.u[k] = -1;
-            ch.nd[k] = 0;
-            if (e < ES) {
-                const uint32_t wd = e >> 5;
-                const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
-                ch.u[k] = ld_stream(col + r.base + e, pol);
-                ch.nd[k] = r.nd;
-            }
-        }
+        for (int k = 0; k < 4 * G; ++k) item[k] = (uint32_t)(u[k] - vb);
+        warp_append_mask<4 * G>(s, w, wn, msk, item, true);
     }
 }
 
-// Expand the batch: each warp takes chunks w, w + 16, ...; the columns of its
-// next chunk are in flight while the current one is probed and relaxed (two
-// chunks of memory-level parallelism per warp).
 __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t NL, uint32_t NLC, uint32_t ES,
                             uint32_t &wn) {
     const int w = threadIdx.x >> 5;
@@ -191,23 +195,35 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
     const uint32_t ntot = NLC + (ES + kLong - 1) / kLong;
     const int64_t vb = s.R.v_begin;
     uint32_t hits = 0;
-    uint32_t c = (uint32_t)w;
-    Chunk1 a;
-    if (c < ntot) load_chunk1(bb, col, pol, NL, NLC, ES, c, lane, below, a);
-    while (c < ntot) {
-        const uint32_t cn = c + kWarps;
-        Chunk1 b;
-        if (cn < ntot) load_chunk1(bb, col, pol, NL, NLC, ES, cn, lane, below, b);
+    for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
+        if (c < NLC) {
+            long_chunk<kLongG>(s, bb, kp, col, pol, NL, c, lane, hcs, vb, wn, hits);
+            continue;
+        }
+        // short rows: packed edge space, coalesced 4-B column loads
+        int32_t u[4];
+        uint32_t nd[4];
+        const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const uint32_t e = c0 + 32u * k + lane;
+            u[k] = -1;
+            nd[k] = 0;
+            if (e < ES) {
+                const uint32_t wd = e >> 5;
+                const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
+                u[k] = ld_stream(col + r.base + e, pol);
+                nd[k] = r.nd;
+            }
+        }
         uint32_t msk;
-        relax_bfs1<4>(s, kp, hcs, a.u, a.nd, msk, hits);
+        relax_bfs1<4>(s, kp, hcs, u, nd, msk, hits);
         if (__any_sync(kFull, msk != 0)) {
             uint32_t item[4];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(a.u[k] - vb);
+            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(u[k] - vb);
             warp_append_mask<4>(s, w, wn, msk, item, true);
         }
-        a = b;
-        c = cn;
     }
     if (kp.hub_n) {
         hits = __reduce_add_sync(kFull, hits);
@@ -222,7 +238,7 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     BatchBuf &bb = s.bb[0];
     const int tid = threadIdx.x;
     const bool hub = kp.hub_chunks > 0;
-    if (hub && tid == 0) {
+    if (hub && tid == 0 && !(kp.hub_dbg & 2)) {
         s.hub_par ^= 1u;              // parity of this batch's copy (read by all threads after the scan's barriers)
         s.hub_rnd++;
         hub_copy_issue(s, kp);
@@ -277,7 +293,7 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     // one scan for four counts: long chunks [40,64) | long rows [30,40) | short edges [10,30) | short rows [0,10)
     const bool lng = deg >= kLong;
     const uint32_t lo = (uint32_t)(b & 3);
-    const uint32_t nch = lng ? (uint32_t)((deg + lo + kLong - 1) / kLong) : 0u;
+    const uint32_t nch = lng ? (uint32_t)((deg + lo + kLong * kLongG - 1) / (kLong * kLongG)) : 0u;
     const int64_t x = lng ? (((int64_t)nch << 40) | (1ll << 30)) : ((deg << 10) | (deg > 0 ? 1 : 0));
     int64_t ex;
     const int64_t tot = block_exscan(s, x, ex);
@@ -308,7 +324,7 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) de += __shfl_xor_sync(kFull, de, o);
     if ((tid & 31) == 0 && de) atomicAdd(&s.c_edges, de);
-    if (hub) hub_copy_wait(s, s.hub_par ^ 1u);             // this batch's bounds have landed
+    if (hub && !(kp.hub_dbg & 2)) hub_copy_wait(s, s.hub_par ^ 1u);             // this batch's bounds have landed
     __syncthreads();
     if (NLC + ES > 0) {
         const int w = tid >> 5;
@@ -317,6 +333,6 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
-    if (hub) hub_refresh(s, kp, cta, s.hub_rnd);
+    if (hub && !(kp.hub_dbg & 1)) hub_refresh(s, kp, cta);
 }
 

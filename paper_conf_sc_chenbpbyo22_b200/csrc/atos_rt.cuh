@@ -301,6 +301,7 @@ struct KParams {
     int32_t hub_n;           // BFS hub bounds: vertex ids [0, hub_n) covered (multiple of 2048; 0 = off)
     int32_t hub_chunks;      // hub_n / 128
     int32_t bfs1;            // single-rank BFS: the lean expansion of atos_bfs1.cuh (else the generic one)
+    int32_t hub_dbg;         // experiment (ATOS_HUB_DBG): 1 no re-scan, 2 no copy, 4 no per-edge test
     int32_t split;           // BFS row pieces: edges per piece (0 = off), see kPieceBit
     int32_t combine;         // PR sender-side residual combining (multi-rank)
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained

@@ -86,7 +86,11 @@ struct alignas(16) BRec {
     uint32_t nd;     // candidate depth of the row's targets (popped depth + 1)
     uint32_t len;    // long row: edges in the row (piece); short row: unused
 };
-constexpr int kLong = 128;           // rows of >= kLong edges are expanded as aligned 128-edge chunks
+constexpr int kLong = 128;           // rows of >= kLong edges are expanded as aligned chunks of kLongG x 128 edges
+#ifndef ATOS_LONGG
+#define ATOS_LONGG 2
+#endif
+constexpr int kLongG = ATOS_LONGG;
 constexpr int kLcv = 4096;           // long chunks whose row is precomputed per batch
 
 struct BatchBuf {
