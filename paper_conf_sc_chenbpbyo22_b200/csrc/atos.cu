@@ -24,7 +24,7 @@
 using namespace atos;
 
 constexpr int kColPad = 4;   // column arrays end with 4 spare entries (16-B loads of a row's last edges)
-constexpr int64_t kHubAutoN = 1 << 21;   // hub bounds cover the top 2^21 ids by default (16 KB of shared memory)
+constexpr int64_t kHubAutoN = 3 << 19;   // hub bounds cover the top 1.5 M ids by default (12 KB of shared memory)
 constexpr int64_t kHubMaxN = 1 << 22;
 
 
@@ -304,7 +304,7 @@ template <typename F>
 static cudaError_t kernel_setup_fn(F *fn, int &occ, size_t smem, int want) {
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    const double need_kb = (double)want * ((double)(smem + sizeof(KParams) + 1024 + 1024) / 1024.0);   // + static + reserved
+    const double need_kb = (double)want * ((double)(smem + 1024) / 1024.0);   // + 1 KB reserved per CTA
     int pct = (int)(need_kb / 228.0 * 100.0) + 1;
     pct = pct > 100 ? 100 : pct;
     e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct);

@@ -100,6 +100,10 @@ __device__ __forceinline__ void hub_mbar_init(Smem &s) {   // one thread, before
     s.hub_rnd = 0;
 }
 
+__device__ __forceinline__ void hub_fill_unknown(Smem &s, const KParams &kp) {   // (ATOS_HUB_DBG without the copy)
+    for (int i = threadIdx.x; i < kp.hub_chunks; i += kThreads) hub_base(s)[i] = 255;
+}
+
 // Relax N edges per lane (u[k] < 0: no edge): hub-bound test, filter probe,
 // red.min + filter store on the probe's verdict (relax_red; duplicates are
 // skipped at pop by the pending bit, the flush fences before publishing).
@@ -158,13 +162,13 @@ __device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KP
     const BRec r = bb.rec[kThreads - 1 - li];
     const uint32_t lo = (uint32_t)(r.base & 3);
     const int64_t a = r.base - lo;
-    const uint32_t rel0 = (c - bb.lq0[li]) * (uint32_t)(kLong * G) + 4u * lane;   // edge offset from a
+    const uint32_t rel0 = (c - bb.lq0[li]) * (uint32_t)(kCh1 * G) + 4u * lane;   // edge offset from a
     const uint32_t end = lo + r.len;
     int32_t u[4 * G];
     uint32_t nd[4 * G];
 #pragma unroll
     for (int g = 0; g < G; ++g) {
-        const uint32_t rel = rel0 + (uint32_t)kLong * g;
+        const uint32_t rel = rel0 + (uint32_t)kCh1 * g;
         int4 v = make_int4(-1, -1, -1, -1);
         if (rel < end) v = ld_stream4(col + a + rel, pol);   // may read <= 3 entries past the row (padded array)
         u[4 * g + 0] = (rel >= lo && rel < end) ? v.x : -1;
@@ -192,7 +196,7 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
     const uint8_t *const hcs = hub_base(s);
     const uint64_t pol = policy_evict_first();
     const uint32_t below = lane == 31 ? 0xFFFFFFFEu : (((2u << lane) - 1u) & ~1u);
-    const uint32_t ntot = NLC + (ES + kLong - 1) / kLong;
+    const uint32_t ntot = NLC + (ES + kCh1 - 1) / kCh1;
     const int64_t vb = s.R.v_begin;
     uint32_t hits = 0;
     for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
@@ -203,7 +207,7 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
         // short rows: packed edge space, coalesced 4-B column loads
         int32_t u[4];
         uint32_t nd[4];
-        const uint32_t c0 = (c - NLC) * (uint32_t)kLong;
+        const uint32_t c0 = (c - NLC) * (uint32_t)kCh1;
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
             const uint32_t e = c0 + 32u * k + lane;
@@ -293,7 +297,7 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     // one scan for four counts: long chunks [40,64) | long rows [30,40) | short edges [10,30) | short rows [0,10)
     const bool lng = deg >= kLong;
     const uint32_t lo = (uint32_t)(b & 3);
-    const uint32_t nch = lng ? (uint32_t)((deg + lo + kLong * kLongG - 1) / (kLong * kLongG)) : 0u;
+    const uint32_t nch = lng ? (uint32_t)((deg + lo + kCh1 * kLongG - 1) / (kCh1 * kLongG)) : 0u;
     const int64_t x = lng ? (((int64_t)nch << 40) | (1ll << 30)) : ((deg << 10) | (deg > 0 ? 1 : 0));
     int64_t ex;
     const int64_t tot = block_exscan(s, x, ex);

@@ -43,7 +43,7 @@ constexpr int kApPr = 1;
 constexpr int kU = ATOS_KU;          // edges per lane in flight
 constexpr int kChunk = 32 * kU;      // edges per warp chunk
 #ifndef ATOS_WOUT
-#define ATOS_WOUT 256
+#define ATOS_WOUT 128
 #endif
 constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
@@ -77,7 +77,7 @@ template <> struct AppTraits<kApPr> { static constexpr int kMsgBytes = 16; };
 // row holding edge 32w, nzslot[] maps compacted rows to batch slots.  A lane's row
 // is then rowmap[w] + popc(bm[w] & lanes (0, lane]) -- one word per 32 edges
 // instead of a per-lane binary search over the batch offsets.
-constexpr int kBitW = 2048;
+constexpr int kBitW = 1024;
 constexpr int64_t kBitE = (int64_t)kBitW * 32;
 
 // One row of a popped batch in the single-rank BFS expansion (atos_bfs1.cuh).
@@ -86,30 +86,36 @@ struct alignas(16) BRec {
     uint32_t nd;     // candidate depth of the row's targets (popped depth + 1)
     uint32_t len;    // long row: edges in the row (piece); short row: unused
 };
-constexpr int kLong = 128;           // rows of >= kLong edges are expanded as aligned chunks of kLongG x 128 edges
+constexpr int kLong = 64;            // rows of >= kLong edges are expanded as aligned chunks of kLongG x kCh1 edges
+constexpr int kCh1 = 128;            // edges per warp chunk in atos_bfs1.cuh (32 lanes x 4)
 #ifndef ATOS_LONGG
-#define ATOS_LONGG 2
+#define ATOS_LONGG 1
 #endif
 constexpr int kLongG = ATOS_LONGG;
-constexpr int kLcv = 4096;           // long chunks whose row is precomputed per batch
+constexpr int kLcv = 2048;           // long chunks whose row is precomputed per batch
 
 struct BatchBuf {
-    uint32_t v[kThreads];          // local vertex ids
-    uint64_t val[kThreads];        // depth (BFS) or delta bits (PR)
-    int64_t beg[kThreads];         // row begin (offset into col)
-    int64_t off[kThreads + 1];     // exclusive prefix of edge counts
-    uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
+    uint32_t v[kThreads];          // popped items (vertex ids / row pieces)
     uint32_t chunk_next;           // next unclaimed edge chunk
     int32_t use_bm;                // the edge map below is valid for this batch
     uint32_t bm[kBitW];
     uint16_t rowmap[kBitW];
-    uint16_t nzslot[kThreads];
-    // single-rank BFS expansion (atos_bfs1.cuh): one 16-B record per row -- short
-    // rows at [0, NZ) in edge-map order, long rows at [kThreads - NL, kThreads) --,
-    // the long-row chunk -> row map and the first chunk of every long row
-    BRec rec[kThreads];
-    uint16_t lcv[kLcv];
-    uint32_t lq0[kThreads];
+    // The two expansions use disjoint per-row tables (a launch runs one of them),
+    // so they share storage: shared memory not used here is L1 for the probes.
+    union {
+        struct {                   // generic expansion (PageRank, multi-rank, BFS options off the default)
+            uint64_t val[kThreads];        // depth (BFS) or delta bits (PR)
+            int64_t beg[kThreads];         // row begin (offset into col)
+            int64_t off[kThreads + 1];     // exclusive prefix of edge counts
+            uint16_t chunk_v[kChunkMap + 1];  // vertex (batch index) holding the first edge of each chunk
+            uint16_t nzslot[kThreads];
+        };
+        struct {                   // single-rank BFS expansion (atos_bfs1.cuh): one 16-B record per row --
+            BRec rec[kThreads];            // short rows at [0, NZ) in edge-map order, long rows at
+            uint16_t lcv[kLcv];            // [kThreads - NL, kThreads) --, the long-chunk -> row map and
+            uint32_t lq0[kThreads];        // the first chunk of every long row
+        };
+    };
 };
 
 // batch slot holding edge e (e = 32 * w + lane) from the edge map
@@ -1425,6 +1431,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
     if (APP == kApBfs && !MULTI && tid == 0) hub_mbar_init(s);   // hub bounds: TMA completion barrier
+    if (APP == kApBfs && !MULTI && (kp.hub_dbg & 2)) hub_fill_unknown(s, kp);
     __syncthreads();
     constexpr bool multi = MULTI;
     const bool coordinator = multi && s.R.rank == 0 && cta == 0;
