@@ -977,6 +977,7 @@ static KParams make_params(atos_graph *g) {
     kp.bfs1 = g->p == 1 && kp.filter && kp.relax_red && !std::getenv("ATOS_BFS_V1");
     if (!kp.bfs1) kp.hub_n = kp.hub_chunks = 0;
     if (const char *e = std::getenv("ATOS_HUB_DBG")) kp.hub_dbg = std::atoi(e);   // experiment
+    if (const char *e = std::getenv("ATOS_TIMELINE")) kp.timeline_ns = std::atoll(e) * 1000;   // experiment
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
     kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices

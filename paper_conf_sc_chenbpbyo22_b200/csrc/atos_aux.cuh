@@ -50,6 +50,10 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         R.ctrl->ring_base.v = R.ctrl->tail.v;
+        if (kp.timeline_ns) {
+            R.ctrl->tl_t0 = globaltimer();
+            for (int k = 0; k < kTimeline; ++k) R.ctrl->tl_edges[k] = R.ctrl->tl_batches[k] = R.ctrl->tl_pops[k] = 0;
+        }
         if (src < R.v_begin || src >= R.v_end) continue;
         R.depth[src] = dw_make(0);
         filt_put_fresh(R.filt, src, 0u);
@@ -97,6 +101,14 @@ __global__ void bump_tail_kernel(KParams kp) {
 // ring stays consistent for the next solve (slots marked consumed; T and F
 // advanced by the same amount).  One CTA.
 __global__ void fixup_kernel(KParams kp) {
+    if (kp.timeline_ns && threadIdx.x == 0) {   // experiment: print the work timeline of rank 0
+        const Ctrl *c = kp.ranks[0].ctrl;
+        printf("TIMELINE bucket_us %lld:", (long long)(kp.timeline_ns / 1000));
+        for (int k = 0; k < kTimeline; ++k)
+            if (c->tl_batches[k]) printf(" [%d %llu %llu %llu]", k, (unsigned long long)c->tl_edges[k],
+                                         (unsigned long long)c->tl_batches[k], (unsigned long long)c->tl_pops[k]);
+        printf("\n");
+    }
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         const uint64_t h = R.ctrl->head.v, t = R.ctrl->tail.v;

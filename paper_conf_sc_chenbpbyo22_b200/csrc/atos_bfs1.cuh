@@ -45,7 +45,7 @@ __device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
 // graph once per batch of every worker: warp gw scans chunks gw + GW * j (up to
 // 4 per warp with 2^21 hubs and 296 workers), loads first, then the reductions.
 // Called after the warp's expansion, where it waits for the batch-end barrier.
-__device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, int cta) {
+__device__ __forceinline__ void hub_refresh(Smem &s, const KParams &kp, int cta) {
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t C = (uint32_t)kp.hub_n >> 7;            // (the array's padding stays 255)
     const uint32_t GW = (uint32_t)kp.ctas_per_rank * kWarps;
@@ -63,7 +63,9 @@ __device__ __forceinline__ void hub_refresh(const Smem &s, const KParams &kp, in
             const uint32_t c = cb + GW * j;
             const uint32_t m = max(max(x[j] & 255u, (x[j] >> 8) & 255u), max((x[j] >> 16) & 255u, x[j] >> 24));
             const uint32_t cm = __reduce_max_sync(kFull, m);
-            if (lane == 0 && c < C) s.R.hcb[c] = (uint8_t)cm;
+            // store only a tighter bound than this worker's copy holds (most re-scans
+            // change nothing; stores into the array every worker copies from cost)
+            if (lane == 0 && c < C && cm < hub_base(s)[c]) s.R.hcb[c] = (uint8_t)cm;
         }
     }
 }
@@ -328,6 +330,15 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) de += __shfl_xor_sync(kFull, de, o);
     if ((tid & 31) == 0 && de) atomicAdd(&s.c_edges, de);
+    if (kp.timeline_ns && (tid & 31) == 0 && de) {        // experiment: work timeline of the solve
+        const uint64_t b = (globaltimer() - R.ctrl->tl_t0) / (uint64_t)kp.timeline_ns;
+        const int k = b < (uint64_t)kTimeline ? (int)b : kTimeline - 1;
+        atomicAdd((unsigned long long *)&R.ctrl->tl_edges[k], de);
+        if (tid == 0) {
+            atomicAdd((unsigned long long *)&R.ctrl->tl_batches[k], 1ull);
+            atomicAdd((unsigned long long *)&R.ctrl->tl_pops[k], (unsigned long long)B);
+        }
+    }
     if (hub && !(kp.hub_dbg & 2)) hub_copy_wait(s, s.hub_par ^ 1u);             // this batch's bounds have landed
     __syncthreads();
     if (NLC + ES > 0) {

@@ -212,6 +212,8 @@ __device__ __forceinline__ uint64_t pack(uint32_t hi, uint32_t lo) { return ((ui
 // ---------------------------------------------------------------------------
 // control block: every counter on its own 128-byte line
 // ---------------------------------------------------------------------------
+constexpr int kTimeline = 64;
+
 struct alignas(128) Line {
     uint64_t v;
     uint64_t pad_[15];
@@ -238,6 +240,9 @@ struct Ctrl {
     Line limit;                  // discrete mode: queue snapshot this launch may pop up to
     Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_hits, st_waves;
     Line st_busy_ns, st_batches;
+    // experiment (ATOS_TIMELINE=<bucket us>): edges / batches / pops started per time bucket of a solve
+    uint64_t tl_t0;
+    uint64_t tl_edges[kTimeline], tl_batches[kTimeline], tl_pops[kTimeline];
 };
 
 // Per-rank device view.  One per rank served by the grid (virtual ranks: many).
@@ -302,6 +307,7 @@ struct KParams {
     int32_t hub_chunks;      // hub_n / 128
     int32_t bfs1;            // single-rank BFS: the lean expansion of atos_bfs1.cuh (else the generic one)
     int32_t hub_dbg;         // experiment (ATOS_HUB_DBG): 1 no re-scan, 2 no copy, 4 no per-edge test
+    int64_t timeline_ns;     // experiment (ATOS_TIMELINE): bucket width of the per-solve work timeline (0 = off)
     int32_t split;           // BFS row pieces: edges per piece (0 = off), see kPieceBit
     int32_t combine;         // PR sender-side residual combining (multi-rank)
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained
