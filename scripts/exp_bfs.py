@@ -28,7 +28,8 @@ def run(g, srcs, reps=4, **cfg):
         util = st["busy_ns"] / (st["grid_ctas"] * st["n_ranks"] * st["ms_worker"] * 1e6)
         rows.append(dict(ms=st["ms_worker"], gteps=m / st["ms_worker"] / 1e6, pops=st["pops"] / nr,
                          edges=st["edges"] / m, util=util, batches=st["batches"], idle=st["idle_polls"], iters=st["iterations"],
-                         hub=st["hub_hits"] / max(1, st["edges"])))
+                         hub=st["hub_hits"] / max(1, st["edges"]), msgs=st["msgs_sent"],
+                         mpp=st["msgs_sent"] / max(1, st["packets_sent"])))
     G.free()
     agg = {k: sum(r[k] for r in rows) / len(rows) for k in rows[0]}
     return agg
