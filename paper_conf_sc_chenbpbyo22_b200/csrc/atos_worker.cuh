@@ -322,11 +322,15 @@ __device__ __forceinline__ void warp_append_mask(Smem &s, int w, uint32_t &wn, u
 // copy.  The packet is published (one st.release of its header {seq, count})
 //   aggregation off: after every 32-edge step of the warp (the paper's
 //                    per-warp push, <= 32 messages per packet);
-//   aggregation on : when it is full (agg_batch_msgs) or, at batch end / when
-//                    idle, once its oldest message is agg_max_age_ns old.
-// Messages in open packets are reported as `staged` (termination, section 6).
-// A warp publishes all its open packets before it waits for a free slot, so a
-// waiting warp never holds an unpublished packet that a receiver needs.
+//   aggregation on : when it is full (agg_batch_msgs), when it is older than
+//                    agg_max_age_ns at the next append, and at the latest when
+//                    the warp has finished its share of the batch.
+// A packet never outlives its warp's expansion: a later reservation of the same
+// slot waits for it, and the waiter may be a warp of the same worker that the
+// holder would otherwise wait for at the batch-end barrier.  For the same
+// reason a warp publishes its open packets before it waits for a free slot, so
+// a waiting warp never holds an unpublished packet.  Messages in open packets
+// are reported as `staged` (termination, section 6).
 // ---------------------------------------------------------------------------
 template <int APP> __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn);
 
@@ -444,7 +448,9 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
             __syncwarp();
             if (lane == 0) {
                 s.op_fill[w][d] = fill + take;
-                if (fill + take == pkt || !kp.agg_on) pkt_publish(s, kp, w, d);   // full, or no aggregation
+                if (fill + take == pkt || !kp.agg_on ||                        // full, no aggregation,
+                    globaltimer() - s.op_t0[w][d] >= (uint64_t)kp.agg_age_ns)   // or aged
+                    pkt_publish(s, kp, w, d);
             }
             done += take;
         }
@@ -452,13 +458,13 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
     __syncwarp();
 }
 
-// Whole warp, batch end / idle: publish per the aggregation policy.
+// Whole warp, end of its expansion / batch end / idle: publish everything open.
 template <int APP>
 __device__ void warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t &wn) {
     (void)cta;
     (void)wn;
     (void)batch_end;
-    warp_publish(s, kp, w, kp.agg_on != 0);
+    warp_publish(s, kp, w, false);
 }
 
 // Whole warp: claim the ready prefix (up to kClaim packets) of one inbound
@@ -1230,6 +1236,8 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
             expand_warp_pipe<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         else expand_warp<APP, MULTI>(s, bb, kp, cta, B, E, wn);
+        // a warp's open packets do not outlive its expansion (see warp_append_remote)
+        if constexpr (MULTI) warp_publish(s, kp, w, false);
         // without work keeping, each warp enqueues its discoveries as soon as its
         // chunks are done (one atomic per warp) instead of after the batch barrier
         if (kp.keep == 0 && kp.warp_flush) warp_flush_local(s, w, wn, APP == kApBfs && kp.relax_red);
