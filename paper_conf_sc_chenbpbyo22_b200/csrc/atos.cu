@@ -87,7 +87,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
     cfg->agg_batch_msgs = 256;
-    cfg->agg_max_age_ns = 4000;      // ~the paper's eager WAIT_TIME for BFS
+    cfg->agg_max_age_ns = 0;         // no age flush inside a warp's share of a batch (its end bounds the wait)
     cfg->channel_packets = 1024;
     cfg->watchdog_ms = 60000;
     cfg->rank = 0;

@@ -323,8 +323,8 @@ __device__ __forceinline__ void warp_append_mask(Smem &s, int w, uint32_t &wn, u
 //   aggregation off: after every 32-edge step of the warp (the paper's
 //                    per-warp push, <= 32 messages per packet);
 //   aggregation on : when it is full (agg_batch_msgs), when it is older than
-//                    agg_max_age_ns at the next append, and at the latest when
-//                    the warp has finished its share of the batch.
+//                    agg_max_age_ns (if > 0) at the next append, and at the
+//                    latest when the warp has finished its share of the batch.
 // A packet never outlives its warp's expansion: a later reservation of the same
 // slot waits for it, and the waiter may be a warp of the same worker that the
 // holder would otherwise wait for at the batch-end barrier.  For the same
@@ -449,7 +449,7 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
             if (lane == 0) {
                 s.op_fill[w][d] = fill + take;
                 if (fill + take == pkt || !kp.agg_on ||                        // full, no aggregation,
-                    globaltimer() - s.op_t0[w][d] >= (uint64_t)kp.agg_age_ns)   // or aged
+                    (kp.agg_age_ns > 0 && globaltimer() - s.op_t0[w][d] >= (uint64_t)kp.agg_age_ns))   // or aged
                     pkt_publish(s, kp, w, d);
             }
             done += take;
