@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define ATOS_ABI_VERSION 4
+#define ATOS_ABI_VERSION 5
 #define ATOS_MAX_RANKS 8          /* one NVSwitch box: 8 GPUs */
 #define ATOS_IPC_HANDLE_BYTES 64  /* == sizeof(cudaIpcMemHandle_t) */
 
@@ -151,6 +151,20 @@ typedef struct {
                                  memory returns to the device); 1 = keep it
                                  reserved for the next graph_load in this
                                  process (load/solve/free loops)               */
+    int32_t pq_delta;         /* BFS priority queue (Listing 4's
+                                 DistributedPriorityQueues threshold_delta,
+                                 P:629-639): 0 = FIFO queue (the
+                                 default); > 0 = every rank keeps two rings,
+                                 the current bucket (candidate depth below the
+                                 threshold) and the rest; workers pop only the
+                                 current one, and when it is drained the rings
+                                 swap and the threshold grows by pq_delta.
+                                 1 = level-synchronous order, large = FIFO.
+                                 Needs rank blocks of < 2^30 vertices; ignored
+                                 by PageRank                                  */
+    int32_t pq_threshold;     /* initial threshold (the paper's `threshold`):
+                                 depths below it form the first bucket; 0 =
+                                 pq_delta                                     */
 } atos_config;
 
 /* Per-solve statistics (device counters, summed over the ranks this handle
@@ -171,6 +185,9 @@ typedef struct {
     uint64_t busy_ns;         /* sum over workers of time spent on work (ns)   */
     uint64_t batches;         /* work units (pop batches + packets + chunks)   */
     uint64_t iterations;      /* discrete mode: worker launches in the solve   */
+    uint64_t far_pushes;      /* priority queue: items enqueued into the next
+                                 bucket's ring                                 */
+    uint64_t pq_buckets;      /* priority queue: bucket advances in the solve  */
     int32_t n_ranks;          /* ranks covered by these counters               */
     int32_t grid_ctas;        /* persistent CTAs per rank                      */
 } atos_stats;
@@ -242,6 +259,36 @@ atos_status atos_last_stats(atos_graph *g, atos_stats *stats);
 
 /* Release everything the handle owns.  NULL-safe. */
 atos_status atos_graph_free(atos_graph *g);
+
+/* Queue microbenchmark (Fig. 1, P:809-823 / P:842-911)
+ * on the worker's own ring code (tagged 8-byte slots, u64 monotone indices,
+ * reserve-then-wait pop).  `threads` threads in workers of worker_size threads
+ * (1 thread, 32 warp, 512 CTA) each do `rounds` pushes (op 0), pops
+ * of a prefilled ring (op 1) or push-then-pop pairs (op 2); a worker's leader
+ * reserves fetch_size indices per atomicAdd (the worker's FETCH_SIZE),
+ * or per CAS loop with reserve_cas = 1 (the paper's CAS-queue baseline).
+ * Item of the push (thread t, round r) is t*rounds + r; prefilled item i is i.
+ * popped_out (host or device, threads*rounds entries, or NULL) receives the
+ * item each (thread, round) popped, for conservation checks.  index_base is
+ * the queue's first index (tests start just below 2^32 to cross the 32-bit
+ * slot tags).  ring_cap: pow2; >= threads*rounds for ops 0/1, >= threads for
+ * op 2.  threads: multiple of 512, at most the co-resident thread count
+ * (waiting pops need their producers resident).  *ms_out = device time of the
+ * benchmark kernel (CUDA events).  Errors: ATOS_ERR_INVALID_ARG,
+ * ATOS_ERR_CAPACITY (a push never found its slot free), ATOS_ERR_TIMEOUT (a
+ * pop never saw its item), ATOS_ERR_CUDA / ATOS_ERR_OOM. */
+typedef struct {
+    int32_t worker_size;      /* 1, 32 or 512 threads per worker               */
+    int32_t fetch_size;       /* indices per leader reservation, 1..worker_size */
+    int32_t op;               /* 0 push, 1 pop, 2 push-then-pop                */
+    int32_t rounds;           /* operations per thread (the paper: 10)         */
+    int64_t threads;          /* concurrent threads (multiple of 512)          */
+    uint64_t ring_cap;        /* ring slots (power of two)                     */
+    uint64_t index_base;      /* first queue index                             */
+    int32_t reserve_cas;      /* 1 = CAS-loop reservation                      */
+    int32_t device;           /* CUDA device ordinal                           */
+} atos_qbench_config;
+atos_status atos_queue_bench(const atos_qbench_config *cfg, uint32_t *popped_out, double *ms_out);
 
 /* Thread-local message describing the last failure on this thread. */
 const char *atos_last_error(void);

@@ -9,7 +9,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.environ.get("ATOS_LIB") or os.path.join(PKG, "libatos.so")   # ATOS_LIB: experiment variants
 SOURCES = [os.path.join(CSRC, "atos.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("atos_rt.cuh", "atos_worker.cuh", "atos_aux.cuh")] + \
+DEPS = SOURCES + [os.path.join(CSRC, f) for f in ("atos_rt.cuh", "atos_worker.cuh", "atos_aux.cuh", "atos_bfs1.cuh", "atos_qbench.cuh")] + \
     [os.path.join(ROOT, "include", "atos.h")]
 
 NVCC_FLAGS = [

@@ -56,6 +56,8 @@ class Config(ctypes.Structure):
         ("discrete", ctypes.c_int32),
         ("pr_combine", ctypes.c_int32),
         ("pool_retain", ctypes.c_int32),
+        ("pq_delta", ctypes.c_int32),
+        ("pq_threshold", ctypes.c_int32),
     ]
 
 
@@ -74,12 +76,28 @@ class Stats(ctypes.Structure):
         ("busy_ns", ctypes.c_uint64),
         ("batches", ctypes.c_uint64),
         ("iterations", ctypes.c_uint64),
+        ("far_pushes", ctypes.c_uint64),
+        ("pq_buckets", ctypes.c_uint64),
         ("n_ranks", ctypes.c_int32),
         ("grid_ctas", ctypes.c_int32),
     ]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class QBenchConfig(ctypes.Structure):
+    _fields_ = [
+        ("worker_size", ctypes.c_int32),
+        ("fetch_size", ctypes.c_int32),
+        ("op", ctypes.c_int32),
+        ("rounds", ctypes.c_int32),
+        ("threads", ctypes.c_int64),
+        ("ring_cap", ctypes.c_uint64),
+        ("index_base", ctypes.c_uint64),
+        ("reserve_cas", ctypes.c_int32),
+        ("device", ctypes.c_int32),
+    ]
 
 
 class AtosError(RuntimeError):
@@ -108,6 +126,7 @@ _SIGS = [
     ("atos_sync", ctypes.c_int, [_P]),
     ("atos_last_stats", ctypes.c_int, [_P, ctypes.POINTER(Stats)]),
     ("atos_graph_free", ctypes.c_int, [_P]),
+    ("atos_queue_bench", ctypes.c_int, [ctypes.POINTER(QBenchConfig), _P, ctypes.POINTER(ctypes.c_double)]),
     ("atos_last_error", ctypes.c_char_p, []),
     ("atos_version", ctypes.c_int32, []),
 ]
@@ -279,6 +298,25 @@ class Graph:
 
     def __exit__(self, *a):
         self.free()
+
+
+QB_OPS = {"push": 0, "pop": 1, "push_then_pop": 2}
+
+
+def queue_bench(worker_size: int, op: str, threads: int, rounds: int = 10, fetch_size: Optional[int] = None,
+                ring_cap: Optional[int] = None, index_base: int = 0, reserve_cas: bool = False,
+                popped: bool = False, device: int = 0):
+    """atos_queue_bench: returns (ms, popped items or None)."""
+    total = threads * rounds
+    if ring_cap is None:
+        ring_cap = 1 << max(10, (total - 1).bit_length())
+    c = QBenchConfig(worker_size, fetch_size or worker_size, QB_OPS[op], rounds, threads, ring_cap, index_base,
+                     1 if reserve_cas else 0, device)
+    out = np.empty(total, dtype=np.uint32) if popped else None
+    ms = ctypes.c_double(0)
+    _check(load().atos_queue_bench(ctypes.byref(c), out.ctypes.data_as(_P) if out is not None else None,
+                                   ctypes.byref(ms)))
+    return ms.value, out
 
 
 # function-style aliases with the C names

@@ -20,6 +20,9 @@
 #include "../../include/atos.h"
 #include "atos_aux.cuh"
 #include "atos_worker.cuh"
+namespace atos {
+#include "atos_qbench.cuh"
+}
 
 using namespace atos;
 
@@ -100,6 +103,8 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->split_edges = -1;
     cfg->pr_combine = 0;
     cfg->pool_retain = 0;
+    cfg->pq_threshold = 0;
+    cfg->pq_delta = 0;
     return ATOS_OK;
 }
 
@@ -136,14 +141,15 @@ static bool valid_cfg(const atos_config &c) {
            (c.split_edges == 0 || c.split_edges == -1 ||
             (c.split_edges >= 256 && c.split_edges <= (1 << 20) && pow2(c.split_edges))) &&
            (c.pr_combine == 0 || c.pr_combine == 1) && (c.pool_retain == 0 || c.pool_retain == 1) &&
-           (c.discrete == 0 || (c.discrete == 1 && c.n_ranks == 1 && c.virtual_ranks == 1));
+           (c.discrete == 0 || (c.discrete == 1 && c.n_ranks == 1 && c.virtual_ranks == 1)) &&
+           c.pq_threshold >= 0 && c.pq_delta >= 0;
 }
 
 // ---------------------------------------------------------------------------
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, filt, hcb, rank, res, ring, in_hdr, in_pay, free_m, parent, ghost, total;
+    size_t ctrl, depth, filt, hcb, rank, res, ring, ring2, in_hdr, in_pay, free_m, parent, ghost, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -161,6 +167,7 @@ struct Shape {
     double ring_factor;
     int combine;       // PR ghost residuals allocated (n_ranks > 1 && pr_combine)
     int hub_chunks;    // BFS hub bounds array (single rank)
+    int pq;            // priority queue (N1): second ring allocated
 };
 
 static Layout make_layout(const Shape &S, const int64_t *part, int r) {
@@ -177,6 +184,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.rank = o;    o = al(o + (size_t)L.n_r * 8);
     L.res = o;     o = al(o + (size_t)L.n_r * 8);
     L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
+    L.ring2 = o;   o = al(o + (S.pq ? (size_t)L.ring_cap * 8 : 0));
     const bool multi = S.p > 1;
     L.in_hdr = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
     L.in_pay = o;  o = al(o + (multi ? (size_t)S.p * S.cp * S.pkt * 16 : 0));
@@ -206,7 +214,7 @@ struct LocalRank {
     int64_t *row_ptr = nullptr;
     int32_t *col = nullptr;
     int64_t m_r = 0;
-    uint64_t snap[10] = {0};  // stat counters after the previous solve
+    uint64_t snap[12] = {0};  // stat counters after the previous solve
 };
 
 struct atos_graph {
@@ -336,6 +344,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     d.pr_q = pr_q_of(L.n_r);
     d.pr_ghost = (g->p > 1 && g->S.combine) ? (double *)(b + L.ghost) : nullptr;
     d.ring = (uint64_t *)(b + L.ring);
+    d.ring2 = g->S.pq ? (uint64_t *)(b + L.ring2) : nullptr;
     d.ring_cap = L.ring_cap;
     d.ctrl = (Ctrl *)(b + L.ctrl);
     const size_t cp = (size_t)g->S.cp, pkt = (size_t)g->S.pkt;
@@ -541,7 +550,7 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
     else atos_partition_balanced(n, n_ranks, pt.data());
     Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs,
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
-            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0};
+            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
     *bytes_out = make_layout(S, pt.data(), rank).total;
     return ATOS_OK;
 }
@@ -757,6 +766,10 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     } else {
         atos_partition_balanced(n, g->p, g->part.data());
     }
+    if (cfg.pq_delta > 0)      // priority queue items carry a bucket tag in bit 30
+        for (int r = 0; r < g->p; ++r)
+            if (g->part[r + 1] - g->part[r] >= ((int64_t)1 << 30))
+                return fail(ATOS_ERR_INVALID_ARG, "priority queue: rank blocks must hold < 2^30 vertices");
 
     // row offsets at partition boundaries (host copies of a few entries)
     const bool rp_dev = is_device_ptr(row_ptr);
@@ -800,7 +813,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
     g->grid = cpr * g->n_local;
     g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, cpr,
-                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0};
+                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
 
     if (cfg.stream) {
         g->stream = (cudaStream_t)cfg.stream;
@@ -875,6 +888,22 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
                                                        (uint64_t *)(me.arena + me.L.free_m), nfree,
                                                        (uint64_t)(g->S.cp / nsub_for(g->p, g->S.cp)));
+        if (g->S.pq)
+            init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring2), me.L.ring_cap,
+                                                           nullptr, 0, 1);
+        if (const char *e = std::getenv("ATOS_TEST_RING_BASE")) {
+            // test-only: start every ring index at this value (tests start just below
+            // 2^32 so that the 32-bit slot tags wrap during the solves)
+            const uint64_t base = std::strtoull(e, nullptr, 0);
+            for (int q = 0; q < (g->S.pq ? 2 : 1); ++q)
+                qbench_init_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + (q ? me.L.ring2 : me.L.ring)),
+                                                               me.L.ring_cap, base, 0);
+            Ctrl *c = (Ctrl *)(me.arena + me.L.ctrl);
+            for (uint64_t *f : {&c->head.v, &c->tail.v, &c->finished.v, &c->ring_base.v, &c->pq_head.v, &c->pq_tail.v,
+                                &c->pq_fin.v, &c->pq_base.v})
+                CU(cudaMemcpyAsync(f, &base, 8, cudaMemcpyHostToDevice, g->stream));
+            CU(cudaStreamSynchronize(g->stream));
+        }
         CU(cudaGetLastError());
     }
     unsigned long long bad = 0;
@@ -987,6 +1016,15 @@ static KParams make_params(atos_graph *g) {
     kp.static_chunks = std::getenv("ATOS_DYNAMIC_CHUNKS") ? 0 : 1;
     if (const char *f = std::getenv("ATOS_TEST_FAULT"))   // test-only fault injection (T6 error paths)
         kp.fault = std::strcmp(f, "capacity") == 0 ? kFaultCapacity : std::strcmp(f, "timeout") == 0 ? kFaultTimeout : 0;
+    if (g->S.pq) {
+        // priority queue (N1): no work keeping (a kept chain would bypass the
+        // buckets) and no early reservation (it is ring-0 only)
+        kp.pq = 1;
+        kp.pq_delta = (uint32_t)g->cfg.pq_delta;
+        kp.pq_th0 = (uint32_t)(g->cfg.pq_threshold > 0 ? g->cfg.pq_threshold : g->cfg.pq_delta);
+        kp.keep = 0;
+        kp.early = 0;
+    }
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
     kp.epoch = g->epoch;
@@ -1116,7 +1154,7 @@ static atos_status read_ctrl(atos_graph *g, int lr, Ctrl &c) {
 }
 
 // Wait for the enqueued solve, check device error flags, fill g->last.
-static constexpr int kSnap = 10;
+static constexpr int kSnap = 12;
 
 // Back to the state graph_load left: control blocks, rings, channel headers and
 // free mirrors re-initialised, statistics snapshots cleared.  Single process only.
@@ -1129,6 +1167,9 @@ static atos_status reset_queues(atos_graph *g) {
         init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring), me.L.ring_cap,
                                                        (uint64_t *)(me.arena + me.L.free_m), nfree,
                                                        (uint64_t)(g->S.cp / nsub_for(g->p, g->S.cp)));
+        if (g->S.pq)
+            init_arena_kernel<<<1024, 256, 0, g->stream>>>((uint64_t *)(me.arena + me.L.ring2), me.L.ring_cap,
+                                                           nullptr, 0, 1);
         CU(cudaGetLastError());
         std::memset(me.snap, 0, sizeof(me.snap));
     }
@@ -1157,7 +1198,7 @@ static atos_status finish_solve(atos_graph *g) {
         if (c.error.v && !err) err = c.error.v;
         const uint64_t now[kSnap] = {c.st_pops.v, c.st_edges.v, c.st_pushes.v, c.st_msgs.v,
                                      c.st_packets.v, c.st_idle.v, c.st_hub_hits.v, c.st_busy_ns.v,
-                                     c.st_batches.v, c.st_waves.v};
+                                     c.st_batches.v, c.st_waves.v, c.st_far.v, c.pq_state.v};
         uint64_t *sn = g->loc[lr].snap;
         st.pops += now[0] - sn[0];
         st.edges += now[1] - sn[1];
@@ -1169,6 +1210,8 @@ static atos_status finish_solve(atos_graph *g) {
         st.busy_ns += now[7] - sn[7];
         st.batches += now[8] - sn[8];
         if (g->cfg.discrete) st.iterations += now[9] - sn[9];
+        st.far_pushes += now[10] - sn[10];
+        st.pq_buckets += now[11] - sn[11];
         std::memcpy(sn, now, sizeof(now));
     }
     st.bytes_sent = st.msgs_sent * (uint64_t)(app == kApBfs ? AppTraits<kApBfs>::kMsgBytes
@@ -1302,6 +1345,7 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     KParams kp;
     atos_status s = begin_solve(g, kp);
     if (s != ATOS_OK) return s;
+    kp.pq = 0;                     // the priority queue orders BFS by depth only
     kp.alpha = alpha;
     kp.eps = eps;
     kp.eps_g = eps / (double)g->p;
@@ -1338,4 +1382,78 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     s = finish_solve(g);
     if (stats) *stats = g->last;
     return s;
+}
+
+// ---------------------------------------------------------------------------
+// queue microbenchmark (Fig. 1) on the worker's ring code
+// ---------------------------------------------------------------------------
+extern "C" atos_status atos_queue_bench(const atos_qbench_config *c, uint32_t *popped_out, double *ms_out) {
+    if (!c || !ms_out) return fail(ATOS_ERR_INVALID_ARG, "queue_bench: NULL argument");
+    auto pow2 = [](uint64_t x) { return x > 0 && (x & (x - 1)) == 0; };
+    if (!(c->worker_size == 1 || c->worker_size == 32 || c->worker_size == kThreads) || c->fetch_size < 1 ||
+        c->fetch_size > c->worker_size || c->rounds < 1 || c->op < 0 || c->op > 2 || c->threads < kThreads ||
+        c->threads % kThreads != 0 || !pow2(c->ring_cap) || (c->reserve_cas != 0 && c->reserve_cas != 1))
+        return fail(ATOS_ERR_INVALID_ARG, "queue_bench: bad configuration");
+    const uint64_t total = (uint64_t)c->threads * (uint64_t)c->rounds;
+    if (c->op != kQPushPop && c->ring_cap < total)
+        return fail(ATOS_ERR_INVALID_ARG, "queue_bench: push / pop alone need ring_cap >= threads * rounds");
+    if (c->op == kQPushPop && c->ring_cap < (uint64_t)c->threads)
+        return fail(ATOS_ERR_INVALID_ARG, "queue_bench: push-then-pop needs ring_cap >= threads");
+    CU(cudaSetDevice(c->device));
+    int sms = 0, per_sm = 0;
+    CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device));
+    CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, qbench_kernel, kThreads, 0));
+    if (c->threads > (int64_t)sms * per_sm * kThreads)
+        return fail(ATOS_ERR_INVALID_ARG, "queue_bench: threads exceed the co-resident limit (%lld)",
+                    (long long)sms * per_sm * kThreads);
+    cudaStream_t st;
+    CU(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    uint64_t *ring = nullptr;
+    Ctrl *ctrl = nullptr;
+    uint32_t *pop = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    atos_status rs = ATOS_OK;
+    auto done = [&](atos_status r) {
+        cudaStreamSynchronize(st);
+        cudaFree(ring); cudaFree(ctrl); cudaFree(pop);
+        if (e0) cudaEventDestroy(e0);
+        if (e1) cudaEventDestroy(e1);
+        cudaStreamDestroy(st);
+        return r;
+    };
+    auto ck = [&](cudaError_t e, const char *what) {
+        if (e != cudaSuccess && rs == ATOS_OK)
+            rs = fail(e == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA, "queue_bench: %s: %s", what,
+                      cudaGetErrorString(e));
+        return e == cudaSuccess;
+    };
+    if (!ck(cudaMalloc(&ring, c->ring_cap * 8), "ring") || !ck(cudaMalloc(&ctrl, sizeof(Ctrl)), "ctrl") ||
+        (popped_out && !is_device_ptr(popped_out) && !ck(cudaMalloc(&pop, total * 4), "popped")) ||
+        !ck(cudaEventCreate(&e0), "event") || !ck(cudaEventCreate(&e1), "event"))
+        return done(rs);
+    uint32_t *pdev = popped_out ? (is_device_ptr(popped_out) ? popped_out : pop) : nullptr;
+    const uint64_t prefill = c->op == kQPop ? total : 0;
+    ck(cudaMemsetAsync(ctrl, 0, sizeof(Ctrl), st), "memset");
+    qbench_init_kernel<<<1024, 256, 0, st>>>(ring, c->ring_cap, c->index_base, prefill);
+    Ctrl h{};
+    h.head.v = c->index_base;
+    h.tail.v = c->index_base + prefill;
+    ck(cudaMemcpyAsync(&ctrl->head.v, &h.head.v, 8, cudaMemcpyHostToDevice, st), "head");
+    ck(cudaMemcpyAsync(&ctrl->tail.v, &h.tail.v, 8, cudaMemcpyHostToDevice, st), "tail");
+    QBenchArgs a{ring, c->ring_cap, ctrl, pdev, c->worker_size, c->fetch_size, c->rounds, c->op, c->reserve_cas,
+                 c->index_base};
+    ck(cudaEventRecord(e0, st), "record");
+    qbench_kernel<<<(unsigned)(c->threads / kThreads), kThreads, 0, st>>>(a);
+    ck(cudaGetLastError(), "launch");
+    ck(cudaEventRecord(e1, st), "record");
+    if (pdev && pdev != popped_out) ck(cudaMemcpyAsync(popped_out, pdev, total * 4, cudaMemcpyDeviceToHost, st), "copy");
+    uint64_t err = 0;
+    ck(cudaMemcpyAsync(&err, &ctrl->error.v, 8, cudaMemcpyDeviceToHost, st), "error");
+    ck(cudaStreamSynchronize(st), "sync");
+    float ms = 0;
+    ck(cudaEventElapsedTime(&ms, e0, e1), "elapsed");
+    *ms_out = ms;
+    if (rs == ATOS_OK && err == kErrCapacity) rs = fail(ATOS_ERR_CAPACITY, "queue_bench: ring capacity exceeded");
+    if (rs == ATOS_OK && err) rs = fail(ATOS_ERR_TIMEOUT, "queue_bench: a pop never saw its item");
+    return done(rs);
 }

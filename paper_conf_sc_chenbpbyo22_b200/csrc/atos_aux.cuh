@@ -50,6 +50,8 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
         R.ctrl->ring_base.v = R.ctrl->tail.v;
+        R.ctrl->pq_base.v = R.ctrl->pq_tail.v;
+        R.ctrl->pq_k0.v = R.ctrl->pq_state.v;      // priority queue: first bucket of this solve
         if (kp.timeline_ns) {
             R.ctrl->tl_t0 = globaltimer();
             for (int k = 0; k < kTimeline; ++k) R.ctrl->tl_edges[k] = R.ctrl->tl_batches[k] = R.ctrl->tl_pops[k] = 0;
@@ -57,13 +59,14 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
         if (src < R.v_begin || src >= R.v_end) continue;
         R.depth[src] = dw_make(0);
         filt_put_fresh(R.filt, src, 0u);
-        const uint64_t idx = R.ctrl->tail.v;
-        uint64_t *p = &R.ring[idx & (R.ring_cap - 1)];
+        const int q = kp.pq ? (int)(R.ctrl->pq_state.v & 1) : 0;   // the current bucket's ring
+        const uint64_t idx = *q_tail(R, q);
+        uint64_t *p = &q_slots(R, q)[idx & (R.ring_cap - 1)];
         if (!slot_free_for(*p, idx)) { R.ctrl->error.v = kErrCapacity; return; }
         __threadfence();
         *p = pack(lo32(idx + 1), (uint32_t)(src - R.v_begin));
         __threadfence();
-        R.ctrl->tail.v = idx + 1;
+        *q_tail(R, q) = idx + 1;
     }
 }
 
@@ -111,17 +114,19 @@ __global__ void fixup_kernel(KParams kp) {
     }
     for (int lr = 0; lr < kp.n_local; ++lr) {
         const RankDev &R = kp.ranks[lr];
-        const uint64_t h = R.ctrl->head.v, t = R.ctrl->tail.v;
-        if (h > t) {
-            for (uint64_t idx = t + threadIdx.x; idx < h; idx += blockDim.x)
-                R.ring[idx & (R.ring_cap - 1)] = pack(lo32(idx + R.ring_cap), 0u);
+        for (int q = 0; q < (R.ring2 ? 2 : 1); ++q) {      // both rings with the priority queue
+            const uint64_t h = *q_head(R, q), t = *q_tail(R, q);
+            if (h > t) {
+                for (uint64_t idx = t + threadIdx.x; idx < h; idx += blockDim.x)
+                    q_slots(R, q)[idx & (R.ring_cap - 1)] = pack(lo32(idx + R.ring_cap), 0u);
+            }
+            __syncthreads();
+            if (threadIdx.x == 0 && h > t) {
+                *q_tail(R, q) = h;
+                *q_fin(R, q) += h - t;
+            }
+            __syncthreads();
         }
-        __syncthreads();
-        if (threadIdx.x == 0 && h > t) {
-            R.ctrl->tail.v = h;
-            R.ctrl->finished.v += h - t;
-        }
-        __syncthreads();
     }
 }
 

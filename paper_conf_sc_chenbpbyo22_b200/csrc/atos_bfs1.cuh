@@ -184,8 +184,9 @@ __device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KP
     relax_bfs1<4 * G>(s, kp, hcs, u, nd, msk, hits);
     if (__any_sync(kFull, msk != 0)) {
         uint32_t item[4 * G];
+        const uint32_t tag = r.nd >= s.pq_th ? kFarBit : 0u;     // priority queue (N1): far bucket
 #pragma unroll
-        for (int k = 0; k < 4 * G; ++k) item[k] = (uint32_t)(u[k] - vb);
+        for (int k = 0; k < 4 * G; ++k) item[k] = (uint32_t)(u[k] - vb) | tag;
         warp_append_mask<4 * G>(s, w, wn, msk, item, true);
     }
 }
@@ -227,7 +228,7 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
         if (__any_sync(kFull, msk != 0)) {
             uint32_t item[4];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) item[k] = (uint32_t)(u[k] - vb);
+            for (int k = 0; k < 4; ++k) item[k] = pq_tag((uint32_t)(u[k] - vb), nd[k], s.pq_th);
             warp_append_mask<4>(s, w, wn, msk, item, true);
         }
     }
@@ -287,13 +288,13 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
         int64_t pex;
         const int64_t ptot = block_exscan(s, (int64_t)npc, pex);
         if (tid == 0) {
-            s.b64[2] = atomicAdd((unsigned long long *)&R.ctrl->tail.v, (unsigned long long)ptot);
+            s.b64[2] = atomicAdd((unsigned long long *)q_tail(R, s.pq_q), (unsigned long long)ptot);
             s.c_pushes += (unsigned long long)ptot;
         }
         __syncthreads();
         const uint64_t pbase = s.b64[2] + (uint64_t)pex;
         for (uint32_t i = 0; i < npc; ++i)
-            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
+            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], ring_base_q(s, s.pq_q), s.pq_q);
     }
     for (int i = tid; i < kBitW; i += kThreads) bb.bm[i] = 0u;
     // one scan for four counts: long chunks [40,64) | long rows [30,40) | short edges [10,30) | short rows [0,10)

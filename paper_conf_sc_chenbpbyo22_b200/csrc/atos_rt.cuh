@@ -237,9 +237,14 @@ struct Ctrl {
     Line out_reserve[kMaxRanks * kMaxSub]; // packets reserved on sub-channel (this -> d, k) at [d * nsub + k]
     Line in_cursor[kMaxRanks * kMaxSub];   // next packet to consume on sub-channel (s -> this, k)
     Line ring_base;              // tail at the start of the current solve
+    // priority queue (Listing 4's DistributedPriorityQueues,
+    // P:629-639): a second ring with its own head / tail / finished counters.
+    // pq_state counts bucket advances (monotone across solves): the CURRENT ring
+    // is pq_state & 1, the threshold th0 + (pq_state - pq_k0) * delta.
+    Line pq_head, pq_tail, pq_fin, pq_base, pq_state, pq_k0;
     Line limit;                  // discrete mode: queue snapshot this launch may pop up to
     Line st_pops, st_edges, st_pushes, st_msgs, st_packets, st_idle, st_hub_hits, st_waves;
-    Line st_busy_ns, st_batches;
+    Line st_busy_ns, st_batches, st_far;
     // experiment (ATOS_TIMELINE=<bucket us>): edges / batches / pops started per time bucket of a solve
     uint64_t tl_t0;
     uint64_t tl_edges[kTimeline], tl_batches[kTimeline], tl_pops[kTimeline];
@@ -263,6 +268,7 @@ struct RankDev {
     int64_t pr_q;                // PR slot spreading: n_r / 8 (0 = identity), see pr_slot
     // local ring (own memory)
     uint64_t *ring;
+    uint64_t *ring2;             // priority queue: the second ring (same capacity); NULL = FIFO
     uint64_t ring_cap;           // power of two
     Ctrl *ctrl;                  // own control block
     Ctrl *peer_ctrl[kMaxRanks];  // control block of every rank (own included)
@@ -314,6 +320,9 @@ struct KParams {
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming
     int32_t fault;           // test-only fault injection (FaultKind), raised by rank 0 CTA 0 at start
+    int32_t pq;              // BFS priority queue (N1): items of depth >= threshold go to the other ring
+    uint32_t pq_th0;         // initial threshold (depths < pq_th0 form the first bucket)
+    uint32_t pq_delta;       // threshold_delta: the threshold grows by this at every bucket advance
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;
@@ -329,6 +338,24 @@ struct KParams {
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ bool slot_full_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx + 1); }
 __device__ __forceinline__ bool slot_free_for(uint64_t slot, uint64_t idx) { return hi32(slot) == lo32(idx); }
+
+// The two rings of a rank (ring 1 exists only with the priority queue, N1):
+// slots, reservation head, push tail (T) and finished count (F) of ring q.
+__host__ __device__ __forceinline__ uint64_t *q_slots(const RankDev &R, int q) { return q ? R.ring2 : R.ring; }
+__host__ __device__ __forceinline__ uint64_t *q_head(const RankDev &R, int q) { return q ? &R.ctrl->pq_head.v : &R.ctrl->head.v; }
+__host__ __device__ __forceinline__ uint64_t *q_tail(const RankDev &R, int q) { return q ? &R.ctrl->pq_tail.v : &R.ctrl->tail.v; }
+__host__ __device__ __forceinline__ uint64_t *q_fin(const RankDev &R, int q) { return q ? &R.ctrl->pq_fin.v : &R.ctrl->finished.v; }
+__host__ __device__ __forceinline__ uint64_t *q_base(const RankDev &R, int q) { return q ? &R.ctrl->pq_base.v : &R.ctrl->ring_base.v; }
+
+// Priority-queue item tag: a discovered vertex whose candidate depth is at or
+// above the current threshold goes to the other ring (rank-local ids < 2^30 in
+// this mode; pieces, bit 31, are never tagged).
+constexpr uint32_t kFarBit = 0x40000000u;
+constexpr uint32_t kNoTh = 0xFFFFFFFFu;      // threshold when the priority queue is off
+__device__ __forceinline__ uint32_t pq_tag(uint32_t item, uint32_t nd, uint32_t th) {
+    return nd >= th ? (item | kFarBit) : item;
+}
+__device__ __forceinline__ bool pq_is_far(uint32_t item) { return (item & (0x80000000u | kFarBit)) == kFarBit; }
 
 // PR state placement: local id i lives at slot (i mod 8) * q + i / 8 (q = n_r / 8,
 // identity on the tail), so that ids adjacent after degree relabeling -- the

@@ -138,7 +138,13 @@ struct alignas(16) Smem {
     uint64_t op_pidx[kWarps][kMaxRanks];   // its index in the warp's sub-channel
     uint64_t op_t0[kWarps][kMaxRanks];     // globaltimer when it was opened
     int64_t wsum[kWarps];
-    uint64_t res_lo, res_hi;       // outstanding ring reservation
+    uint64_t res_lo, res_hi;       // outstanding ring reservation (ring 0)
+    uint64_t res2_lo, res2_hi;     // priority queue: outstanding reservation on ring 1
+    uint64_t ring2_base;           // ring 1 tail at the start of this solve
+    uint64_t pq_st;                // priority queue: pq_state read at the last pop
+    uint32_t pq_th;                // current threshold (kNoTh: FIFO, nothing is far)
+    int32_t pq_q;                  // current ring (pq_state & 1; 0 without the priority queue)
+    int32_t pop_q;                 // ring the current batch was popped from
     uint64_t limit;                // discrete mode: this launch pops indices < limit
     uint64_t ring_base;            // ring tail at the start of this solve
     uint64_t b64[4];
@@ -155,7 +161,7 @@ struct alignas(16) Smem {
     uint32_t hub_par, hub_rnd;
     uint64_t in_cc;
     uint32_t in_off[33];
-    unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches;
+    unsigned long long c_pops, c_edges, c_pushes, c_msgs, c_packets, c_idle, c_hub, c_busy, c_batches, c_far;
 #ifdef ATOS_PROF
     unsigned long long prof[10];
 #endif
@@ -247,8 +253,12 @@ __device__ __forceinline__ int upper_vertex(const BatchBuf &bb, int lo, int hi, 
 // ---------------------------------------------------------------------------
 // local ring pushes
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ void ring_store(const RankDev &R, uint64_t idx, uint32_t item, uint64_t base) {
-    uint64_t *p = &R.ring[idx & (R.ring_cap - 1)];
+__device__ __forceinline__ uint64_t &res_lo_q(Smem &s, int q) { return q ? s.res2_lo : s.res_lo; }
+__device__ __forceinline__ uint64_t &res_hi_q(Smem &s, int q) { return q ? s.res2_hi : s.res_hi; }
+__device__ __forceinline__ uint64_t ring_base_q(const Smem &s, int q) { return q ? s.ring2_base : s.ring_base; }
+
+__device__ __forceinline__ void ring_store(const RankDev &R, uint64_t idx, uint32_t item, uint64_t base, int q = 0) {
+    uint64_t *p = &q_slots(R, q)[idx & (R.ring_cap - 1)];
     uint32_t spins = 0;
     // every index below the solve's base was consumed or retired, so slots of the
     // first lap of this solve are free without looking; later laps check the tag
@@ -259,12 +269,51 @@ __device__ __forceinline__ void ring_store(const RankDev &R, uint64_t idx, uint3
     st_relaxed_gpu(p, pack(lo32(idx + 1), item));
 }
 
+// Consumer of index idx: read its slot (published iff slot_full_for) and, once
+// the item is taken, hand the slot to the producer of idx + cap.
+__device__ __forceinline__ uint64_t ring_read(const uint64_t *ring, uint64_t cap, uint64_t idx) {
+    return ld_relaxed_gpu(&ring[idx & (cap - 1)]);
+}
+__device__ __forceinline__ void ring_release(uint64_t *ring, uint64_t cap, uint64_t idx) {
+    st_relaxed_gpu(&ring[idx & (cap - 1)], pack(lo32(idx + cap), 0u));
+}
+
 // Whole warp: push wout[w][0..wn) with one leader atomic.
 __device__ void warp_flush_local(Smem &s, int w, uint32_t &wn, bool fence) {
     __syncwarp();
     const uint32_t cnt = wn;
     if (cnt == 0) return;
     const int lane = threadIdx.x & 31;
+    if (s.pq_th != kNoTh) {
+        // priority queue (N1): far-tagged items go to the other ring
+        const int q = s.pq_q;
+        uint32_t nf = 0;
+        for (uint32_t i0 = 0; i0 < cnt; i0 += 32)
+            nf += __popc(__ballot_sync(kFull, i0 + lane < cnt && pq_is_far(s.wout[w][i0 + lane])));
+        unsigned long long bn = 0, bf = 0;
+        if (lane == 0) {
+            if (cnt > nf) bn = atomicAdd((unsigned long long *)q_tail(s.R, q), (unsigned long long)(cnt - nf));
+            if (nf) bf = atomicAdd((unsigned long long *)q_tail(s.R, q ^ 1), (unsigned long long)nf);
+            atomicAdd(&s.c_far, (unsigned long long)nf);
+        }
+        bn = __shfl_sync(kFull, bn, 0);
+        bf = __shfl_sync(kFull, bf, 0);
+        if (fence) fence_acq_rel_gpu();
+        for (uint32_t i0 = 0; i0 < cnt; i0 += 32) {
+            const uint32_t i = i0 + lane;
+            const uint32_t it = i < cnt ? s.wout[w][i] : 0u;
+            const bool far = i < cnt && pq_is_far(it);
+            const uint32_t mf = __ballot_sync(kFull, far), mn = __ballot_sync(kFull, i < cnt && !far);
+            if (far) ring_store(s.R, bf + __popc(mf & lanemask_lt()), it & ~kFarBit, ring_base_q(s, q ^ 1), q ^ 1);
+            else if (i < cnt) ring_store(s.R, bn + __popc(mn & lanemask_lt()), it, ring_base_q(s, q), q);
+            bf += __popc(mf);
+            bn += __popc(mn);
+        }
+        if (lane == 0) atomicAdd(&s.c_pushes, (unsigned long long)cnt);
+        wn = 0;
+        __syncwarp();
+        return;
+    }
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd((unsigned long long *)&s.R.ctrl->tail.v, (unsigned long long)cnt);
     base = __shfl_sync(kFull, base, 0);
@@ -532,6 +581,7 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                             const uint32_t ndw = dw_make(hi32(m[j]));
                             pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
                             if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(m[j]));
+                            ul[j] = pq_tag(ul[j], hi32(m[j]), s.pq_th);
                         }
                     }
                 } else {
@@ -651,6 +701,7 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                     const uint32_t ndw = dw_make(hi32(msg));
                     pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
                     if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(msg));
+                    ul[j] = pq_tag(ul[j], hi32(msg), s.pq_th);
                 } else {
                     const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
                     ul[j] = msg.x;
@@ -748,6 +799,7 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
     double *const res = R.pr_res;
     const uint64_t pol = policy_evict_first();
     const uint32_t nch = (uint32_t)((E + kChunk - 1) / kChunk);
+    const uint32_t th = s.pq_th;       // BFS priority queue threshold (kNoTh: off)
     int jprev = 0;
     uint32_t cs = (uint32_t)(threadIdx.x >> 5);   // static schedule: chunks w, w + 16, ...
     for (;;) {
@@ -840,7 +892,7 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
 #pragma unroll
                 for (int k = 0; k < kU; ++k) {
                     msk |= (imp[k] ? 1u : 0u) << k;
-                    item[k] = (uint32_t)(u[k] - vb);
+                    item[k] = pq_tag((uint32_t)(u[k] - vb), nd[k], th);
                 }
                 warp_append_mask<kU>(s, w, wn, msk, item, kp.relax_red);
             } else {
@@ -848,7 +900,7 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                 for (int k = 0; k < kU; ++k) {
                     const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
                     if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
-                    warp_append_local(s, w, wn, loc, (uint32_t)(u[k] - vb));
+                    warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(u[k] - vb), nd[k], th));
                     const bool rem = imp[k] && !loc;
                     const int d = rem ? owner_of(R, u[k]) : 0;
                     warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
@@ -984,7 +1036,7 @@ __device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, 
     for (int k = 0; k < kPU; ++k) {
         const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
         if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
-        warp_append_local(s, w, wn, loc, (uint32_t)(st.u[k] - vb));
+        warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(st.u[k] - vb), st.nd[k], s.pq_th));
         if constexpr (MULTI) {
             const bool rem = imp[k] && !loc;
             const int d = rem ? owner_of(R, st.u[k]) : 0;
@@ -1061,7 +1113,7 @@ __device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta
 #pragma unroll
         for (int k = 0; k < kPU; ++k) {
             msk |= (imp[k] ? 1u : 0u) << k;
-            item[k] = (uint32_t)(st.u[k] - vb);
+            item[k] = pq_tag((uint32_t)(st.u[k] - vb), st.nd[k], s.pq_th);
         }
         warp_append_mask<kPU>(s, w, wn, msk, item, kp.relax_red);
     } else {
@@ -1069,7 +1121,7 @@ __device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta
         for (int k = 0; k < kPU; ++k) {
             const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
             if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
-            warp_append_local(s, w, wn, loc, (uint32_t)(st.u[k] - vb));
+            warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(st.u[k] - vb), st.nd[k], s.pq_th));
             const bool rem = imp[k] && !loc;
             const int d = rem ? owner_of(R, st.u[k]) : 0;
             warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
@@ -1176,13 +1228,13 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         int64_t pex;
         const int64_t ptot = block_exscan(s, (int64_t)npc, pex);
         if (tid == 0) {
-            s.b64[2] = atomicAdd((unsigned long long *)&R.ctrl->tail.v, (unsigned long long)ptot);
+            s.b64[2] = atomicAdd((unsigned long long *)q_tail(R, s.pq_q), (unsigned long long)ptot);
             s.c_pushes += (unsigned long long)ptot;
         }
         __syncthreads();
         const uint64_t pbase = s.b64[2] + (uint64_t)pex;
         for (uint32_t i = 0; i < npc; ++i)
-            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], s.ring_base);
+            ring_store(R, pbase + i, kPieceBit | ((i + 1) << 16) | bb.v[tid], ring_base_q(s, s.pq_q), s.pq_q);
     }
     if (kp.prefetch && deg > 0) prefetch_l2_bulk(R.col + bb.beg[tid], (uint64_t)deg * 4);
     if (kp.edge_map)
@@ -1246,6 +1298,59 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
     }
 }
 
+// Priority-queue batch end (N1): the CTA's discoveries go to the current ring
+// (depth below the threshold) or to the other one (far-tagged), one leader
+// atomic per ring.  At most kWarps * kWOut = 4 * kThreads items.
+__device__ void batch_end_pq(Smem &s, const KParams &kp) {
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        uint32_t total = 0;
+        for (int k = 0; k < kWarps; ++k) { s.wpre[k] = total; total += s.wn[k]; }
+        s.wpre[kWarps] = total;
+    }
+    __syncthreads();
+    const uint32_t total = s.wpre[kWarps];
+    constexpr int kPer = kWarps * kWOut / kThreads;
+    static_assert(kWarps * kWOut % kThreads == 0, "items per thread");
+    uint32_t it[kPer];
+    uint32_t nn = 0, nf = 0;
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+        const uint32_t i = (uint32_t)tid + (uint32_t)j * kThreads;
+        it[j] = 0;
+        if (i < total) {
+            int k = 0;
+            while (k + 1 < kWarps && s.wpre[k + 1] <= i) ++k;
+            it[j] = s.wout[k][i - s.wpre[k]];
+            if (pq_is_far(it[j])) ++nf; else ++nn;
+        }
+    }
+    int64_t ex;
+    const int64_t tot = block_exscan(s, ((int64_t)nf << 32) | nn, ex);
+    const int q = s.pq_q;
+    if (tid == 0) {
+        const uint64_t NN = (uint64_t)(tot & 0xFFFFFFFF), NF = (uint64_t)(tot >> 32);
+        s.b64[0] = NN ? atomicAdd((unsigned long long *)q_tail(s.R, q), (unsigned long long)NN) : 0ull;
+        s.b64[1] = NF ? atomicAdd((unsigned long long *)q_tail(s.R, q ^ 1), (unsigned long long)NF) : 0ull;
+        s.c_pushes += NN + NF;
+        s.c_far += NF;
+    }
+    __syncthreads();
+    if (kp.relax_red && total > 0) fence_acq_rel_gpu();   // fire-and-forget relaxations are performed first
+    uint64_t pn = s.b64[0] + (uint64_t)(ex & 0xFFFFFFFF), pf = s.b64[1] + (uint64_t)(ex >> 32);
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+        const uint32_t i = (uint32_t)tid + (uint32_t)j * kThreads;
+        if (i < total) {
+            if (pq_is_far(it[j])) ring_store(s.R, pf++, it[j] & ~kFarBit, ring_base_q(s, q ^ 1), q ^ 1);
+            else ring_store(s.R, pn++, it[j], ring_base_q(s, q), q);
+        }
+    }
+    __syncthreads();
+    if (tid < kWarps) s.wn[tid] = 0;
+    __syncthreads();
+}
+
 // End of a batch: publish remote staging per policy, then enqueue this CTA's
 // local discoveries with one leader atomic -- or keep up to kp.keep of them as
 // the next batch (returned count, already in s.v) when the ring is nearly empty.
@@ -1260,6 +1365,10 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
         __syncthreads();
+    }
+    if (s.pq_th != kNoTh) {         // priority queue (N1): no keeping, split by bucket
+        batch_end_pq(s, kp);
+        return 0;
     }
     if (tid == 0) {
         uint32_t total = 0;
@@ -1323,12 +1432,74 @@ __device__ void report_staged(Smem &s, const KParams &kp) {
 // ---------------------------------------------------------------------------
 // pop from the local ring: reserve-then-wait
 // ---------------------------------------------------------------------------
+// Priority queue (N1; Listing 4 threshold / threshold_delta), leader
+// thread: choose the ring to pop from and make sure a reservation is open on it.
+// The current ring q = pq_state & 1 holds the bucket below the threshold; the
+// other ring collects the discoveries at or above it.  When ring q is drained
+// (every item pushed to it finished: F_q == T_q) while the other ring holds
+// work, the bucket advances: one CAS increments pq_state, which swaps the roles
+// of the rings and raises the threshold by delta.  A reservation left open on
+// the other ring (taken before a swap) is still served: every reserved index
+// must be consumed.
+__device__ void pq_choose(Smem &s, const KParams &kp) {
+    const RankDev &R = s.R;
+    const uint64_t st = ld_relaxed_gpu(&R.ctrl->pq_state.v);
+    const int q = (int)(st & 1);
+    const uint64_t k = st - ld_relaxed_gpu(&R.ctrl->pq_k0.v);
+    const uint64_t th = (uint64_t)kp.pq_th0 + k * (uint64_t)kp.pq_delta;
+    s.pq_st = st;
+    s.pq_q = q;
+    s.pq_th = th < (uint64_t)kNoTh ? (uint32_t)th : kNoTh - 1;
+    s.pop_q = q;
+    if (kp.discrete) {
+        // one launch pops ring q up to the snapshot the step kernel took
+        uint64_t *hd = q_head(R, q);
+        if (s.res_lo == s.res_hi) {
+            const uint64_t h = ld_relaxed_gpu(hd);
+            if (h < s.limit) {
+                uint64_t n = (s.limit - h) / (uint64_t)kp.ctas_per_rank;
+                n = n < 1 ? 1 : (n > (uint64_t)kp.fetch ? (uint64_t)kp.fetch : n);
+                const uint64_t lo = atomicAdd((unsigned long long *)hd, (unsigned long long)n);
+                if (lo < s.limit) {
+                    s.res_lo = lo;
+                    s.res_hi = lo + n < s.limit ? lo + n : s.limit;
+                }
+            }
+        }
+        return;      // (the reservation lives in res_lo / res_hi; its ring is q)
+    }
+    uint64_t &lo = res_lo_q(s, q), &hi = res_hi_q(s, q);
+    if (lo == hi) {
+        const uint64_t t = ld_relaxed_gpu(q_tail(R, q)), h = ld_relaxed_gpu(q_head(R, q));
+        if (t > h) {
+            uint64_t n = (t - h) / (uint64_t)kp.ctas_per_rank;
+            n = n < 1 ? 1 : (n > (uint64_t)kp.fetch ? (uint64_t)kp.fetch : n);
+            lo = atomicAdd((unsigned long long *)q_head(R, q), (unsigned long long)n);
+            hi = lo + n;
+        }
+    }
+    if (lo != hi && slot_full_for(ld_relaxed_gpu(&q_slots(R, q)[lo & (R.ring_cap - 1)]), lo)) return;
+    const int o = q ^ 1;
+    const uint64_t lo2 = res_lo_q(s, o), hi2 = res_hi_q(s, o);
+    if (lo2 != hi2 && slot_full_for(ld_relaxed_gpu(&q_slots(R, o)[lo2 & (R.ring_cap - 1)]), lo2)) {
+        s.pop_q = o;
+        return;
+    }
+    // nothing ready: advance the bucket if ring q is drained and ring o holds work
+    const uint64_t f = ld_acquire_gpu(q_fin(R, q));
+    const uint64_t t = ld_acquire_gpu(q_tail(R, q));
+    if (f == t && ld_relaxed_gpu(q_tail(R, o)) > ld_relaxed_gpu(q_fin(R, o)))
+        atomicCAS((unsigned long long *)&R.ctrl->pq_state.v, (unsigned long long)st, (unsigned long long)(st + 1));
+}
+
 __device__ int pop_batch(Smem &s, const KParams &kp) {
     const RankDev &R = s.R;
     const int tid = threadIdx.x;
     BatchBuf &bb = s.bb[0];
     if (tid == 0) {
-        if (s.res_lo == s.res_hi && kp.discrete) {
+        if (kp.pq) {
+            pq_choose(s, kp);
+        } else if (s.res_lo == s.res_hi && kp.discrete) {
             // discrete mode: reserve with atomicAdd and clip at the launch's snapshot,
             // so every reserved slot is already published; head may overshoot the
             // limit and is set back to it by discrete_step_kernel (a CAS loop here
@@ -1357,13 +1528,18 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
         s.minbad = kThreads;
     }
     __syncthreads();
-    const uint64_t lo = s.res_lo;
-    const uint64_t avail = s.res_hi - lo;
+    // ring of this pop: 0 without the priority queue; in discrete pq mode the
+    // reservation is kept in res_lo/hi for ring pq_q
+    const int q = s.pop_q;
+    const bool dq = kp.pq && kp.discrete;
+    const uint64_t lo = dq ? s.res_lo : res_lo_q(s, q);
+    const uint64_t avail = (dq ? s.res_hi : res_hi_q(s, q)) - lo;
+    uint64_t *const ring = q_slots(R, q);
     const int cnt = (int)(avail < (uint64_t)kp.fetch ? avail : (uint64_t)kp.fetch);
     const uint64_t idx = lo + tid;
     uint64_t slot = 0;
     if (tid < cnt) {
-        slot = ld_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)]);
+        slot = ring_read(ring, R.ring_cap, idx);
         if (!slot_full_for(slot, idx)) atomicMin(&s.minbad, tid);
     }
     __syncthreads();
@@ -1372,10 +1548,13 @@ __device__ int pop_batch(Smem &s, const KParams &kp) {
         // no acquire fence: the vertex state is only accessed through L2 atomics
         // whose address depends on this slot value (see warp_flush_local)
         bb.v[tid] = lo32(slot);
-        st_relaxed_gpu(&R.ring[idx & (R.ring_cap - 1)], pack(lo32(idx + R.ring_cap), 0u));
+        ring_release(ring, R.ring_cap, idx);
     }
     __syncthreads();
-    if (tid == 0) s.res_lo = lo + (uint64_t)B;
+    if (tid == 0) {
+        if (dq) s.res_lo = lo + (uint64_t)B;
+        else res_lo_q(s, q) = lo + (uint64_t)B;
+    }
     return B;
 }
 
@@ -1396,8 +1575,10 @@ __device__ void coordinator_step(Smem &s, const KParams &kp) {
         started = ld_acquire_peer(kp.sys, &R.ctrl->started[lane].v) == kp.epoch;
         const Ctrl *c = R.peer_ctrl[lane];
         F = ld_acquire_peer(kp.sys, &c->finished.v);
+        if (kp.pq) F += ld_acquire_peer(kp.sys, &c->pq_fin.v);
         Rv = ld_acquire_peer(kp.sys, &c->recvd.v);
         T = ld_acquire_peer(kp.sys, &c->tail.v);
+        if (kp.pq) T += ld_acquire_peer(kp.sys, &c->pq_tail.v);
         St = ld_acquire_peer(kp.sys, &c->staged.v);
         S = ld_acquire_peer(kp.sys, &c->sent.v);
     }
@@ -1444,10 +1625,21 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
     if (tid == 0) {
         s.R = kp.ranks[lr];
         s.res_lo = s.res_hi = 0;
+        s.res2_lo = s.res2_hi = 0;
         s.ring_base = s.R.ctrl->ring_base.v;
+        s.ring2_base = s.R.ctrl->pq_base.v;
+        s.pq_q = s.pop_q = 0;
+        s.pq_st = 0;
+        s.pq_th = kNoTh;
+        if (kp.pq) {        // the bucket at the start of the launch (pop_batch re-reads it)
+            const uint64_t st = ld_relaxed_gpu(&s.R.ctrl->pq_state.v);
+            const uint64_t th = (uint64_t)kp.pq_th0 + (st - ld_relaxed_gpu(&s.R.ctrl->pq_k0.v)) * (uint64_t)kp.pq_delta;
+            s.pq_q = s.pop_q = (int)(st & 1);
+            s.pq_th = th < (uint64_t)kNoTh ? (uint32_t)th : kNoTh - 1;
+        }
         s.staged_reported = 0;
         s.wave_valid = 0;
-        s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = 0;
+        s.c_pops = s.c_edges = s.c_pushes = s.c_msgs = s.c_packets = s.c_idle = s.c_hub = s.c_far = 0;
         s.c_busy = s.c_batches = 0;
         s.limit = kp.discrete ? ld_relaxed_gpu(&s.R.ctrl->limit.v) : 0;
 #ifdef ATOS_PROF
@@ -1530,7 +1722,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
                     // before this F update is issued; multi-rank adds a sys fence
                     // because the coordinator reads these counters over NVLink
                     if (multi) fence_peer(kp.sys);
-                    atomicAdd((unsigned long long *)&s.R.ctrl->finished.v, (unsigned long long)B0);  // F last
+                    atomicAdd((unsigned long long *)q_fin(s.R, s.pop_q), (unsigned long long)B0);  // F last
                 }
                 worked = true;
             }
@@ -1554,8 +1746,12 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         if (tid == 0) {
             s.c_idle++;
             if (!multi) {
-                const uint64_t F = ld_acquire_gpu(&s.R.ctrl->finished.v);
-                const uint64_t T = ld_acquire_gpu(&s.R.ctrl->tail.v);
+                // F before T (per ring; F_q <= T_q always): equal sums mean every pushed
+                // item had finished and nothing could produce more
+                uint64_t F = ld_acquire_gpu(&s.R.ctrl->finished.v);
+                if (kp.pq) F += ld_acquire_gpu(&s.R.ctrl->pq_fin.v);
+                uint64_t T = ld_acquire_gpu(&s.R.ctrl->tail.v);
+                if (kp.pq) T += ld_acquire_gpu(&s.R.ctrl->pq_tail.v);
                 if (F == T) st_release_gpu(&s.R.ctrl->done.v, kp.epoch);
             }
         }
@@ -1574,6 +1770,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         atomicAdd((unsigned long long *)&c->st_hub_hits.v, s.c_hub);
         atomicAdd((unsigned long long *)&c->st_busy_ns.v, s.c_busy);
         atomicAdd((unsigned long long *)&c->st_batches.v, s.c_batches);
+        if (s.c_far) atomicAdd((unsigned long long *)&c->st_far.v, s.c_far);
 #ifdef ATOS_PROF
         if (blockIdx.x < 4)
             printf("PROF cta %d chunks %llu col %llu probe %llu atom %llu append %llu (cyc/chunk/warp) | per batch: pop %llu setup %llu expand(t0) %llu end %llu total %llu batches %llu\n",
@@ -1609,10 +1806,20 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) worker_discrete_kernel(c
 __global__ void discrete_step_kernel(const KParams *kpp, cudaGraphConditionalHandle h, int after_launch) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const RankDev &R = kpp->ranks[0];
+    // the ring of this launch: 0, or the current bucket's ring (priority queue)
+    int q = kpp->pq ? (int)(R.ctrl->pq_state.v & 1) : 0;
     // after a launch every index below the old limit was consumed; reservations
     // past it were clipped, so head goes back to the limit
-    if (after_launch && R.ctrl->head.v > R.ctrl->limit.v) R.ctrl->head.v = R.ctrl->limit.v;
-    const uint64_t t = ld_relaxed_gpu(&R.ctrl->tail.v), hd = ld_relaxed_gpu(&R.ctrl->head.v);
+    if (after_launch && *q_head(R, q) > R.ctrl->limit.v) *q_head(R, q) = R.ctrl->limit.v;
+    uint64_t t = ld_relaxed_gpu(q_tail(R, q)), hd = ld_relaxed_gpu(q_head(R, q));
+    if (kpp->pq && t == hd && ld_relaxed_gpu(q_tail(R, q ^ 1)) > ld_relaxed_gpu(q_head(R, q ^ 1))) {
+        // the bucket is drained (a launch retires everything below its limit):
+        // advance it -- the other ring becomes current, the threshold grows by delta
+        R.ctrl->pq_state.v += 1;
+        q ^= 1;
+        t = ld_relaxed_gpu(q_tail(R, q));
+        hd = ld_relaxed_gpu(q_head(R, q));
+    }
     R.ctrl->limit.v = t;
     const bool more = t > hd && ld_relaxed_gpu(&R.ctrl->error.v) == 0;
     if (more) R.ctrl->st_waves.v += 1;          // = worker launches of the solve

@@ -40,7 +40,7 @@ def test_struct_layouts_match_header():
     # compile a probe against the header and compare every field offset
     import subprocess, tempfile
     lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "atos.h"', 'int main(void){']
-    for cname, ct in (("atos_config", atos.Config), ("atos_stats", atos.Stats)):
+    for cname, ct in (("atos_config", atos.Config), ("atos_stats", atos.Stats), ("atos_qbench_config", atos.QBenchConfig)):
         lines.append(f'printf("%zu\\n", sizeof({cname}));')
         for f, _ in ct._fields_:
             lines.append(f'printf("%zu\\n", offsetof({cname}, {f}));')
@@ -51,14 +51,14 @@ def test_struct_layouts_match_header():
         subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), src, "-o", exe])
         got = [int(x) for x in subprocess.check_output([exe]).split()]
     want = []
-    for ct in (atos.Config, atos.Stats):
+    for ct in (atos.Config, atos.Stats, atos.QBenchConfig):
         want.append(ctypes.sizeof(ct))
         want.extend(getattr(ct, f).offset for f, _ in ct._fields_)
     assert got == want
 
 
 def test_version():
-    assert atos.load().atos_version() == 4
+    assert atos.load().atos_version() == 5
 
 
 def test_partition_balanced_matches_definition():
@@ -113,7 +113,18 @@ def test_relabel_and_hub_cache_config_validation():
     for bad in (dict(relabel=3), dict(hub_cache=33), dict(hub_cache=1 << 23), dict(hub_cache=-2),
                 dict(hub_cache=32, virtual_ranks=2), dict(hub_cache=200), dict(split_edges=100), dict(split_edges=128),
                 dict(split_edges=1 << 21), dict(split_edges=-2), dict(pr_combine=2), dict(keep_items=-2), dict(keep_mode=2), dict(discrete=2),
-                dict(discrete=1, virtual_ranks=2), dict(discrete=1, n_ranks=2)):
+                dict(discrete=1, virtual_ranks=2), dict(discrete=1, n_ranks=2), dict(pq_delta=-1), dict(pq_threshold=-1)):
         with pytest.raises(atos.AtosError) as e:
             atos.Graph(rp, col, **bad)
         assert e.value.status == 1, bad
+
+
+def test_queue_bench_rejects_bad_config_without_gpu():
+    for kw in (dict(worker_size=16), dict(fetch_size=64, worker_size=32), dict(threads=1000), dict(rounds=0),
+               dict(ring_cap=1000), dict(op="push", ring_cap=1024)):
+        args = dict(worker_size=32, op="push_then_pop", threads=4096, rounds=10)
+        args.update(kw)
+        with pytest.raises((atos.AtosError, KeyError)) as e:
+            atos.queue_bench(**args)
+        if isinstance(e.value, atos.AtosError):
+            assert e.value.status == 1, kw
