@@ -84,17 +84,18 @@ typedef struct {
                                  persisting carve-out                         */
     double ring_cap_factor;   /* local ring capacity = pow2 >= factor*n_rank   */
     int32_t agg_enabled;      /* communication aggregation: 1 =
-                                 messages accumulate in a per-warp packet per
-                                 destination; 0 = every warp pushes its
-                                 messages after each 32-edge step (Listing 5's
-                                 per-warp push)                    */
+                                 each warp stages its remote messages per
+                                 destination and sends a packet when
+                                 agg_batch_msgs are staged, or at batch end /
+                                 when idle once the oldest staged message is
+                                 agg_max_age_ns old; 0 = every warp sends what
+                                 each 32-edge step produced at once (Listing
+                                 5's per-warp push; packets of <= 32
+                                 messages)                                    */
     int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */
-    int64_t agg_max_age_ns;   /* flush age (the WAIT_TIME), ns of
-                                 %globaltimer: an open packet older than this
-                                 is published at its warp's next append; 0 =
-                                 no age flush.  Packets are always published
-                                 when full and when their warp has finished its
-                                 share of the batch                            */
+    int64_t agg_max_age_ns;   /* flush age (the WAIT_TIME) in ns of
+                                 %globaltimer, checked at batch end and when
+                                 idle                                          */
     int32_t channel_packets;  /* packets per (src->dst) channel ring, pow2    */
     int64_t watchdog_ms;      /* device watchdog per solve; 0 = none           */
     int32_t rank;             /* SPMD: this process's rank                     */

@@ -90,7 +90,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
     cfg->agg_batch_msgs = 256;
-    cfg->agg_max_age_ns = 0;         // no age flush inside a warp's share of a batch (its end bounds the wait)
+    cfg->agg_max_age_ns = 4000;      // ~the paper's eager WAIT_TIME for BFS
     cfg->channel_packets = 1024;
     cfg->watchdog_ms = 60000;
     cfg->rank = 0;
@@ -149,7 +149,7 @@ static bool valid_cfg(const atos_config &c) {
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, filt, hcb, rank, res, ring, ring2, in_hdr, in_pay, free_m, parent, ghost, total;
+    size_t ctrl, depth, filt, hcb, rank, res, ring, ring2, in_hdr, in_pay, free_m, staging, parent, ghost, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -163,7 +163,7 @@ static uint64_t pow2_ceil(uint64_t x) {
 struct Shape {
     int64_t n;
     int p;
-    int cp, pkt, ctas_per_rank, fetch;
+    int cp, pkt, stage_cap, ctas_per_rank, fetch;
     double ring_factor;
     int combine;       // PR ghost residuals allocated (n_ranks > 1 && pr_combine)
     int hub_chunks;    // BFS hub bounds array (single rank)
@@ -189,6 +189,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.in_hdr = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
     L.in_pay = o;  o = al(o + (multi ? (size_t)S.p * S.cp * S.pkt * 16 : 0));
     L.free_m = o;  o = al(o + (multi ? (size_t)S.p * S.cp * 8 : 0));
+    L.staging = o; o = al(o + (multi ? (size_t)S.ctas_per_rank * kWarps * kMaxRanks * S.stage_cap * 16 : 0));
     L.parent = o;  o = al(o + (size_t)S.n * 8);
     L.ghost = o;   o = al(o + (multi && S.combine ? (size_t)S.n * 8 : 0));
     L.total = o;
@@ -203,6 +204,7 @@ static int nsub_for(int p, int cp) {
     return p > 1 ? k : 1;
 }
 
+static int stage_cap_for(int pkt) { return (int)pow2_ceil((uint64_t)std::max(2 * pkt, 64)); }
 
 // ---------------------------------------------------------------------------
 // handle
@@ -348,6 +350,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     d.ring_cap = L.ring_cap;
     d.ctrl = (Ctrl *)(b + L.ctrl);
     const size_t cp = (size_t)g->S.cp, pkt = (size_t)g->S.pkt;
+    d.staging = b + L.staging;
     d.perm = g->d_perm;
     d.inv = g->d_inv;
     for (int s = 0; s < g->p; ++s) {
@@ -548,7 +551,7 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
     std::vector<int64_t> pt(n_ranks + 1);
     if (part) std::copy(part, part + n_ranks + 1, pt.begin());
     else atos_partition_balanced(n, n_ranks, pt.data());
-    Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs,
+    Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs),
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
             cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
     *bytes_out = make_layout(S, pt.data(), rank).total;
@@ -812,7 +815,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     const int cpr = ctas_total / g->n_local;
     if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
     g->grid = cpr * g->n_local;
-    g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, cpr,
+    g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs), cpr,
                  cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
 
     if (cfg.stream) {
@@ -978,6 +981,7 @@ static KParams make_params(atos_graph *g) {
     kp.cp = g->S.cp;
     kp.nsub = nsub_for(g->p, g->S.cp);
     kp.cps = g->S.cp / kp.nsub;
+    kp.stage_cap = g->S.stage_cap;
     kp.agg_on = g->cfg.agg_enabled;
     // auto keeping: only for a persistent single-rank solve on a non-skewed graph
     // (discrete launches chain without bound inside one launch: 87 edges per

@@ -227,7 +227,7 @@ struct Ctrl {
     Line head;                   // local ring: next index to reserve for pop
     Line tail;                   // local ring: next index to reserve for push (T)
     Line finished;               // local ring entries fully processed (F)
-    Line staged;                 // messages written into open (unpublished) packets
+    Line staged;                 // messages sitting in CTA staging buffers
     Line sent;                   // messages published to peer channels (S)
     Line recvd;                  // inbound messages fully processed (R)
     Line done;                   // epoch of the finished solve (set by coordinator)
@@ -279,6 +279,8 @@ struct RankDev {
     unsigned char *out_payload[kMaxRanks];
     uint64_t *free_mirror[kMaxRanks];  // own memory: free tags of packets of channel (this -> d)
     uint64_t *peer_free[kMaxRanks];    // peer memory: s's free_mirror[rank]
+    // CTA-private staging of outbound messages [cta][dst][stage_cap] (own memory)
+    unsigned char *staging;
     // degree relabeling (graph_load); NULL = identity.
     // Vertex ids inside the path are the NEW ids; outputs are mapped back.
     const int32_t *perm;         // [n] old id -> new id
@@ -298,6 +300,7 @@ struct KParams {
     int32_t pkt;             // messages per packet
     int32_t cp;              // packets per channel (pow2) = nsub sub-channels of cps packets
     int32_t nsub, cps;       // sub-channels per channel, packets per sub-channel (pow2)
+    int32_t stage_cap;       // staging capacity per (cta, warp, dst), messages (pow2)
     int32_t agg_on;
     int32_t keep;            // max discovered items a worker keeps for itself (work-keeping chain)
     int32_t keep_always;     // 1: keep whenever <= keep discovered; 0: only when the rank's T - F <= keep

@@ -48,7 +48,6 @@ constexpr int kChunk = 32 * kU;      // edges per warp chunk
 constexpr int kWOut = ATOS_WOUT;     // per-warp local staging (items)
 constexpr int kChunkMap = 1024;      // chunks whose first vertex is precomputed per batch
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr uint32_t kNoPkt = 0xffffffffu;
 
 // BFS row pieces.  A popped row longer than
 // 2 x kp.split edges is cut: the popping worker expands the first kp.split edges
@@ -132,11 +131,8 @@ struct alignas(16) Smem {
     uint32_t wout[kWarps][kWOut];  // per-warp local push staging
     uint32_t wn[kWarps];
     uint32_t wpre[kWarps + 1];
-    // per-warp open packet per destination (remote messages, see warp_append_remote)
-    uint32_t op_slot[kWarps][kMaxRanks];   // channel slot, kNoPkt = none open
-    uint32_t op_fill[kWarps][kMaxRanks];   // messages written into it
-    uint64_t op_pidx[kWarps][kMaxRanks];   // its index in the warp's sub-channel
-    uint64_t op_t0[kWarps][kMaxRanks];     // globaltimer when it was opened
+    uint32_t wst[kWarps][kMaxRanks], wsh[kWarps][kMaxRanks];   // per-warp message staging tail/head
+    uint64_t wt0[kWarps][kMaxRanks];                           // time staging became non-empty
     int64_t wsum[kWarps];
     uint64_t res_lo, res_hi;       // outstanding ring reservation (ring 0)
     uint64_t res2_lo, res2_hi;     // priority queue: outstanding reservation on ring 1
@@ -278,40 +274,46 @@ __device__ __forceinline__ void ring_release(uint64_t *ring, uint64_t cap, uint6
     st_relaxed_gpu(&ring[idx & (cap - 1)], pack(lo32(idx + cap), 0u));
 }
 
+// warp_flush_local with the priority queue (N1): far-tagged items go to the other ring.
+__device__ __noinline__ void warp_flush_local_pq(Smem &s, int w, uint32_t &wn, bool fence) {
+    const uint32_t cnt = wn;
+    const int lane = threadIdx.x & 31;
+    const int q = s.pq_q;
+    uint32_t nf = 0;
+    for (uint32_t i0 = 0; i0 < cnt; i0 += 32)
+        nf += __popc(__ballot_sync(kFull, i0 + lane < cnt && pq_is_far(s.wout[w][i0 + lane])));
+    unsigned long long bn = 0, bf = 0;
+    if (lane == 0) {
+        if (cnt > nf) bn = atomicAdd((unsigned long long *)q_tail(s.R, q), (unsigned long long)(cnt - nf));
+        if (nf) bf = atomicAdd((unsigned long long *)q_tail(s.R, q ^ 1), (unsigned long long)nf);
+        atomicAdd(&s.c_far, (unsigned long long)nf);
+    }
+    bn = __shfl_sync(kFull, bn, 0);
+    bf = __shfl_sync(kFull, bf, 0);
+    if (fence) fence_acq_rel_gpu();
+    for (uint32_t i0 = 0; i0 < cnt; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        const uint32_t it = i < cnt ? s.wout[w][i] : 0u;
+        const bool far = i < cnt && pq_is_far(it);
+        const uint32_t mf = __ballot_sync(kFull, far), mn = __ballot_sync(kFull, i < cnt && !far);
+        if (far) ring_store(s.R, bf + __popc(mf & lanemask_lt()), it & ~kFarBit, ring_base_q(s, q ^ 1), q ^ 1);
+        else if (i < cnt) ring_store(s.R, bn + __popc(mn & lanemask_lt()), it, ring_base_q(s, q), q);
+        bf += __popc(mf);
+        bn += __popc(mn);
+    }
+    if (lane == 0) atomicAdd(&s.c_pushes, (unsigned long long)cnt);
+    wn = 0;
+    __syncwarp();
+}
+
 // Whole warp: push wout[w][0..wn) with one leader atomic.
 __device__ void warp_flush_local(Smem &s, int w, uint32_t &wn, bool fence) {
     __syncwarp();
     const uint32_t cnt = wn;
     if (cnt == 0) return;
     const int lane = threadIdx.x & 31;
-    if (s.pq_th != kNoTh) {
-        // priority queue (N1): far-tagged items go to the other ring
-        const int q = s.pq_q;
-        uint32_t nf = 0;
-        for (uint32_t i0 = 0; i0 < cnt; i0 += 32)
-            nf += __popc(__ballot_sync(kFull, i0 + lane < cnt && pq_is_far(s.wout[w][i0 + lane])));
-        unsigned long long bn = 0, bf = 0;
-        if (lane == 0) {
-            if (cnt > nf) bn = atomicAdd((unsigned long long *)q_tail(s.R, q), (unsigned long long)(cnt - nf));
-            if (nf) bf = atomicAdd((unsigned long long *)q_tail(s.R, q ^ 1), (unsigned long long)nf);
-            atomicAdd(&s.c_far, (unsigned long long)nf);
-        }
-        bn = __shfl_sync(kFull, bn, 0);
-        bf = __shfl_sync(kFull, bf, 0);
-        if (fence) fence_acq_rel_gpu();
-        for (uint32_t i0 = 0; i0 < cnt; i0 += 32) {
-            const uint32_t i = i0 + lane;
-            const uint32_t it = i < cnt ? s.wout[w][i] : 0u;
-            const bool far = i < cnt && pq_is_far(it);
-            const uint32_t mf = __ballot_sync(kFull, far), mn = __ballot_sync(kFull, i < cnt && !far);
-            if (far) ring_store(s.R, bf + __popc(mf & lanemask_lt()), it & ~kFarBit, ring_base_q(s, q ^ 1), q ^ 1);
-            else if (i < cnt) ring_store(s.R, bn + __popc(mn & lanemask_lt()), it, ring_base_q(s, q), q);
-            bf += __popc(mf);
-            bn += __popc(mn);
-        }
-        if (lane == 0) atomicAdd(&s.c_pushes, (unsigned long long)cnt);
-        wn = 0;
-        __syncwarp();
+    if (s.pq_th != kNoTh) {         // priority queue (N1): far-tagged items go to the other ring
+        warp_flush_local_pq(s, w, wn, fence);
         return;
     }
     unsigned long long base = 0;
@@ -362,65 +364,26 @@ __device__ __forceinline__ void warp_append_mask(Smem &s, int w, uint32_t &wn, u
 }
 
 // ---------------------------------------------------------------------------
-// remote messages: one-sided stores straight into the owner's channel
-// (Listing 5 push to the remote queue; aggregation P:995-1065)
-//
-// A warp holds at most one OPEN packet per destination: a slot of its
-// sub-channel in the owner's HBM, reserved with one atomicAdd and filled
-// directly by the lanes' coalesced peer stores as messages arise -- no staging
-// copy.  The packet is published (one st.release of its header {seq, count})
-//   aggregation off: after every 32-edge step of the warp (the paper's
-//                    per-warp push, <= 32 messages per packet);
-//   aggregation on : when it is full (agg_batch_msgs), when it is older than
-//                    agg_max_age_ns (if > 0) at the next append, and at the
-//                    latest when the warp has finished its share of the batch.
-// A packet never outlives its warp's expansion: a later reservation of the same
-// slot waits for it, and the waiter may be a warp of the same worker that the
-// holder would otherwise wait for at the batch-end barrier.  For the same
-// reason a warp publishes its open packets before it waits for a free slot, so
-// a waiting warp never holds an unpublished packet.  Messages in open packets
-// are reported as `staged` (termination, section 6).
+// remote messages: per-warp staging per destination; packets over NVLink
 // ---------------------------------------------------------------------------
+template <int APP>
+__device__ __forceinline__ unsigned char *wstage(const Smem &s, const KParams &kp, int cta, int w, int d) {
+    const size_t slot = (((size_t)cta * kWarps + w) * kMaxRanks + d) * (size_t)kp.stage_cap;
+    return s.R.staging + slot * AppTraits<APP>::kMsgBytes;
+}
+
 template <int APP> __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn);
 
+// Whole warp: publish `cnt` staged messages for dst as one packet.
+// A channel (s -> d) is nsub independent sub-channels (rings of cps packets,
+// own reserve counter and receive cursor); a sending warp always uses the same
+// one, so receivers claiming on different cursors do not serialise on one CAS.
 __device__ __forceinline__ uint32_t sub_slot(const KParams &kp, int k, uint64_t i) {
     return (uint32_t)k * (uint32_t)kp.cps + (uint32_t)(i & (uint64_t)(kp.cps - 1));
 }
 
-// lane 0 only: publish the open packet of (w, d)
-__device__ __forceinline__ void pkt_publish(Smem &s, const KParams &kp, int w, int d) {
-    const RankDev &R = s.R;
-    const uint32_t cnt = s.op_fill[w][d];
-    atomicAdd((unsigned long long *)&R.ctrl->sent.v, (unsigned long long)cnt);   // S before the header
-    // the caller's __syncwarp orders every lane's payload stores before this
-    // release (cumulative), which also orders the S increment
-    st_release_peer(kp.sys, &R.out_hdr[d][s.op_slot[w][d]], pack(lo32(s.op_pidx[w][d] + 1), cnt));
-    s.op_slot[w][d] = kNoPkt;
-    s.op_fill[w][d] = 0;
-    atomicAdd(&s.c_msgs, (unsigned long long)cnt);
-    atomicAdd(&s.c_packets, 1ull);
-}
-
-// Whole warp: publish this warp's open packets -- all of them, or (aged_only)
-// those whose first message is at least agg_max_age_ns old.
-__device__ void warp_publish(Smem &s, const KParams &kp, int w, bool aged_only) {
-    const RankDev &R = s.R;
-    if (R.n_ranks <= 1) return;
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) {
-        const uint64_t now = aged_only ? globaltimer() : 0;
-        for (int d = 0; d < R.n_ranks; ++d)
-            if (s.op_slot[w][d] != kNoPkt && s.op_fill[w][d] > 0 &&
-                (!aged_only || now - s.op_t0[w][d] >= (uint64_t)kp.agg_age_ns))
-                pkt_publish(s, kp, w, d);
-    }
-    __syncwarp();
-}
-
-// Whole warp: open a packet to d (reserve a slot of the warp's sub-channel and
-// wait until the receiver has freed it, consuming inbound packets meanwhile).
 template <int APP>
-__device__ bool pkt_open(Smem &s, const KParams &kp, int cta, int w, int d, uint32_t &wn) {
+__device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int d, uint32_t cnt, uint32_t &wn) {
     const RankDev &R = s.R;
     const int lane = threadIdx.x & 31;
     const int k = (cta * kWarps + w) % kp.nsub;
@@ -429,8 +392,7 @@ __device__ bool pkt_open(Smem &s, const KParams &kp, int cta, int w, int d, uint
     pidx = __shfl_sync(kFull, pidx, 0);
     const uint32_t slot = sub_slot(kp, k, pidx);
     uint64_t t_begin = 0;
-    bool published = false;
-    for (;;) {
+    for (;;) {   // wait for the receiver to free the slot; keep consuming inbound meanwhile
         int st = 0;
         if (lane == 0) {
             const uint64_t f = ld_acquire_peer(kp.sys, &R.free_mirror[d][slot]);
@@ -447,73 +409,94 @@ __device__ bool pkt_open(Smem &s, const KParams &kp, int cta, int w, int d, uint
         st = __shfl_sync(kFull, st, 0);
         if (st == 1) break;
         if (st == 2) return false;
-        if (!published) {           // never wait while holding unpublished packets
-            warp_publish(s, kp, w, false);
-            published = true;
-        }
         warp_inbound<APP>(s, kp, w, wn);
     }
+    const unsigned char *src = wstage<APP>(s, kp, cta, w, d);
+    const uint32_t h = s.wsh[w][d];
+    const uint32_t mask = (uint32_t)(kp.stage_cap - 1);
+    unsigned char *dpay = R.out_payload[d] + (size_t)slot * kp.pkt * AppTraits<APP>::kMsgBytes;
+    for (uint32_t i = lane; i < cnt; i += 32) {     // coalesced one-sided stores into d's HBM
+        const uint32_t q = (h + i) & mask;
+        if constexpr (APP == kApBfs) ((uint64_t *)dpay)[i] = ((const uint64_t *)src)[q];
+        else ((uint4 *)dpay)[i] = ((const uint4 *)src)[q];
+    }
+    // One system-scope release per packet: the warp barrier orders every lane's
+    // payload stores before lane 0's st.release (cumulative), which also orders
+    // the S increment before the header -- S is counted before any receiver can
+    // count the messages in R (termination, section 6).
+    __syncwarp();
     if (lane == 0) {
-        s.op_slot[w][d] = slot;
-        s.op_pidx[w][d] = pidx;
-        s.op_fill[w][d] = 0;
-        s.op_t0[w][d] = globaltimer();
+        atomicAdd((unsigned long long *)&R.ctrl->sent.v, (unsigned long long)cnt);   // S before publish
+        st_release_peer(kp.sys, &R.out_hdr[d][slot], pack(lo32(pidx + 1), cnt));
+        s.wsh[w][d] = h + cnt;
+        if (s.wsh[w][d] == s.wst[w][d]) s.wt0[w][d] = 0;
+        atomicAdd(&s.c_msgs, (unsigned long long)cnt);
+        atomicAdd(&s.c_packets, 1ull);
     }
     __syncwarp();
     return true;
 }
 
-// Whole warp: lanes with pred send a message (dst, v_local at dst, payload)
-// into the open packet of dst, grouped by destination (one group per distinct
-// dst among the warp's lanes), opening / publishing packets as they fill.
+// Whole warp: send full packets (and partial ones when `partial`) for every destination.
+template <int APP>
+__device__ __noinline__ void warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t &wn) {
+    const RankDev &R = s.R;
+    if (R.n_ranks <= 1) return;
+    const uint64_t now = globaltimer();
+    for (int d = 0; d < R.n_ranks; ++d) {
+        if (d == R.rank) continue;
+        for (;;) {
+            __syncwarp();
+            const uint32_t pending = s.wst[w][d] - s.wsh[w][d];
+            if (pending == 0) break;
+            bool go = pending >= (uint32_t)kp.pkt;
+            if (!go && batch_end) {
+                const uint64_t t0 = s.wt0[w][d];
+                go = !kp.agg_on || (t0 != 0 && now - t0 >= (uint64_t)kp.agg_age_ns);
+            }
+            go = __shfl_sync(kFull, go, 0);
+            if (!go) break;
+            const uint32_t cnt = pending < (uint32_t)kp.pkt ? pending : (uint32_t)kp.pkt;
+            if (!warp_send_packet<APP>(s, kp, cta, w, d, cnt, wn)) return;
+        }
+    }
+}
+
+// Whole warp: lanes with pred stage a message (dst, v_local at dst, payload).
 template <int APP>
 __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, int cta, int w, bool pred, int dst,
                                                    uint32_t v_local, uint64_t payload, uint32_t &wn) {
     const RankDev &R = s.R;
-    uint32_t pend = __ballot_sync(kFull, pred);
-    if (pend == 0) return;
+    if (__ballot_sync(kFull, pred) == 0) return;
     const int lane = threadIdx.x & 31;
-    const uint32_t pkt = (uint32_t)kp.pkt;
-    while (pend) {
-        const int d = __shfl_sync(kFull, dst, __ffs(pend) - 1);
-        const uint32_t m = __ballot_sync(kFull, pred && dst == d);
-        pend &= ~m;
-        const uint32_t rk = __popc(m & lanemask_lt());       // this lane's rank in the group
-        uint32_t done = 0;
-        const uint32_t cnt = __popc(m);
-        while (done < cnt) {
+    const uint32_t mask = (uint32_t)(kp.stage_cap - 1);
+    for (int d = 0; d < R.n_ranks; ++d) {
+        const bool mine = pred && dst == d;
+        const uint32_t m = __ballot_sync(kFull, mine);
+        if (m == 0) continue;
+        __syncwarp();
+        if (s.wst[w][d] - s.wsh[w][d] + 32 > (uint32_t)kp.stage_cap) {
+            // full packets out first (keeps room for this row)
+            warp_flush_remote<APP>(s, kp, cta, w, false, wn);
             __syncwarp();
-            if (s.op_slot[w][d] == kNoPkt) {
-                if (!pkt_open<APP>(s, kp, cta, w, d, wn)) return;
-            }
-            const uint32_t fill = s.op_fill[w][d];
-            const uint32_t take = min(pkt - fill, cnt - done);
-            if ((m >> lane) & 1u && rk >= done && rk < done + take) {
-                unsigned char *pay = R.out_payload[d] + (size_t)s.op_slot[w][d] * pkt * AppTraits<APP>::kMsgBytes;
-                const uint32_t i = fill + rk - done;          // coalesced one-sided stores into d's HBM
-                if constexpr (APP == kApBfs) ((uint64_t *)pay)[i] = pack((uint32_t)payload, v_local);
-                else ((uint4 *)pay)[i] = make_uint4(v_local, 0u, (uint32_t)payload, (uint32_t)(payload >> 32));
-            }
-            __syncwarp();
-            if (lane == 0) {
-                s.op_fill[w][d] = fill + take;
-                if (fill + take == pkt || !kp.agg_on ||                        // full, no aggregation,
-                    (kp.agg_age_ns > 0 && globaltimer() - s.op_t0[w][d] >= (uint64_t)kp.agg_age_ns))   // or aged
-                    pkt_publish(s, kp, w, d);
-            }
-            done += take;
         }
+        const uint32_t t = s.wst[w][d];
+        if (mine) {
+            unsigned char *b = wstage<APP>(s, kp, cta, w, d);
+            const uint32_t pos = (t + __popc(m & lanemask_lt())) & mask;
+            if constexpr (APP == kApBfs) ((uint64_t *)b)[pos] = pack((uint32_t)payload, v_local);
+            else ((uint4 *)b)[pos] = make_uint4(v_local, 0u, (uint32_t)payload, (uint32_t)(payload >> 32));
+        }
+        __syncwarp();
+        if (lane == 0) {
+            if (t == s.wsh[w][d]) s.wt0[w][d] = globaltimer();
+            s.wst[w][d] = t + __popc(m);
+        }
+        __syncwarp();
     }
-    __syncwarp();
-}
-
-// Whole warp, end of its expansion / batch end / idle: publish everything open.
-template <int APP>
-__device__ void warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t &wn) {
-    (void)cta;
-    (void)wn;
-    (void)batch_end;
-    warp_publish(s, kp, w, false);
+    // aggregation off: the warp pushes what this 32-edge step produced right away
+    // (Listing 5's per-warp remote push): packets of <= 32 messages
+    if (!kp.agg_on) warp_flush_remote<APP>(s, kp, cta, w, true, wn);
 }
 
 // Whole warp: claim the ready prefix (up to kClaim packets) of one inbound
@@ -1288,8 +1271,6 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
         if (APP == kApBfs && (kp.pipe == 1 || (kp.pipe == 2 && E < 16 * (int64_t)B)))
             expand_warp_pipe<APP, MULTI>(s, bb, kp, cta, B, E, wn);
         else expand_warp<APP, MULTI>(s, bb, kp, cta, B, E, wn);
-        // a warp's open packets do not outlive its expansion (see warp_append_remote)
-        if constexpr (MULTI) warp_publish(s, kp, w, false);
         // without work keeping, each warp enqueues its discoveries as soon as its
         // chunks are done (one atomic per warp) instead of after the batch barrier
         if (kp.keep == 0 && kp.warp_flush) warp_flush_local(s, w, wn, APP == kApBfs && kp.relax_red);
@@ -1301,7 +1282,7 @@ __device__ void process_batch(Smem &s, const KParams &kp, int cta, int B) {
 // Priority-queue batch end (N1): the CTA's discoveries go to the current ring
 // (depth below the threshold) or to the other one (far-tagged), one leader
 // atomic per ring.  At most kWarps * kWOut = 4 * kThreads items.
-__device__ void batch_end_pq(Smem &s, const KParams &kp) {
+__device__ __noinline__ void batch_end_pq(Smem &s, const KParams &kp) {
     const int tid = threadIdx.x;
     if (tid == 0) {
         uint32_t total = 0;
@@ -1416,7 +1397,7 @@ __device__ void report_staged(Smem &s, const KParams &kp) {
     if (threadIdx.x == 0) {
         uint64_t cur = 0;
         for (int w = 0; w < kWarps; ++w)
-            for (int d = 0; d < s.R.n_ranks; ++d) cur += (uint64_t)s.op_fill[w][d];
+            for (int d = 0; d < s.R.n_ranks; ++d) cur += (uint64_t)(s.wst[w][d] - s.wsh[w][d]);
         const uint64_t delta = cur - s.staged_reported;   // mod 2^64
         if (delta != 0) {
             fence_peer(kp.sys);
@@ -1441,7 +1422,7 @@ __device__ void report_staged(Smem &s, const KParams &kp) {
 // of the rings and raises the threshold by delta.  A reservation left open on
 // the other ring (taken before a swap) is still served: every reserved index
 // must be consumed.
-__device__ void pq_choose(Smem &s, const KParams &kp) {
+__device__ __noinline__ void pq_choose(Smem &s, const KParams &kp) {
     const RankDev &R = s.R;
     const uint64_t st = ld_relaxed_gpu(&R.ctrl->pq_state.v);
     const int q = (int)(st & 1);
@@ -1648,7 +1629,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
     }
     if (tid < kWarps) {
         s.wn[tid] = 0;
-        for (int d = 0; d < kMaxRanks; ++d) { s.op_slot[tid][d] = kNoPkt; s.op_fill[tid][d] = 0; s.op_t0[tid][d] = 0; }
+        for (int d = 0; d < kMaxRanks; ++d) { s.wst[tid][d] = s.wsh[tid][d] = 0; s.wt0[tid][d] = 0; }
     }
     if (APP == kApBfs && !MULTI && tid == 0) hub_mbar_init(s);   // hub bounds: TMA completion barrier
     if (APP == kApBfs && !MULTI && (kp.hub_dbg & 2)) hub_fill_unknown(s, kp);
@@ -1784,7 +1765,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
 
 // The persistent worker (one cooperative launch per solve).
 template <int APP, bool MULTI>
-__global__ void __launch_bounds__(kThreads, kMinBlocks) worker_kernel(KParams kp) {
+__global__ void __launch_bounds__(kThreads, kMinBlocks) worker_kernel(const __grid_constant__ KParams kp) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     worker_body<APP, MULTI>(*reinterpret_cast<Smem *>(smem_raw), kp);
 }

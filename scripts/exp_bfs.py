@@ -25,7 +25,7 @@ def run(g, srcs, reps=4, **cfg):
         reached = depth >= 0
         m = int(deg[reached].sum())
         nr = int(reached.sum())
-        util = st["busy_ns"] / (st["grid_ctas"] * st["n_ranks"] * st["ms_worker"] * 1e6)
+        util = st["busy_ns"] / max(1e-9, st["grid_ctas"] * st["n_ranks"] * st["ms_worker"] * 1e6)
         rows.append(dict(ms=st["ms_worker"], gteps=m / st["ms_worker"] / 1e6, pops=st["pops"] / nr,
                          edges=st["edges"] / m, util=util, batches=st["batches"], idle=st["idle_polls"], iters=st["iterations"],
                          hub=st["hub_hits"] / max(1, st["edges"]), msgs=st["msgs_sent"],
