@@ -555,18 +555,31 @@ def virtual_rank_block(G_graph, srcs, cfg, stream, dev):
     g = G_graph
     out = {"what": "same GPU, workers split among the ranks: protocol overhead, not scaling"}
     d = torch.empty(g.n, dtype=torch.int32, device=dev)
+    deg = g.degrees().to(dev)
+    pq = {"what": "N1 priority queue (Listing 4 threshold_delta, P:629-639) vs FIFO: redundant work as in "
+                  "Table III (P:1333-1359) = edges scanned / m_reached and pops / reached, BFS RMAT-24, "
+                  "virtual ranks on this GPU"}
     for vr in (1, 2, 8):
-        H = atos.Graph(g.row_ptr, g.col, g.n, **dict(cfg, virtual_ranks=vr))
-        H.bfs(srcs[0], depth_out=d)
-        H.last_stats()
-        ws = []
-        for s in srcs[:4]:
-            H.bfs(s, depth_out=d)
-            st = H.last_stats()
-            ws.append(st["ms_worker"])
-        out[f"bfs_rmat24_vr{vr}_ms"] = statistics.median(ws)
-        out[f"bfs_rmat24_vr{vr}_msgs_per_solve"] = st["msgs_sent"]
-        H.free()
+        for delta in (0, 1):
+            H = atos.Graph(g.row_ptr, g.col, g.n, **dict(cfg, virtual_ranks=vr, pq_delta=delta))
+            H.bfs(srcs[0], depth_out=d)
+            H.last_stats()
+            ws, ed, po = [], [], []
+            for s in srcs[:4]:
+                H.bfs(s, depth_out=d)
+                st = H.last_stats()
+                ws.append(st["ms_worker"])
+                reached = d >= 0
+                ed.append(st["edges"] / max(1, int(deg[reached].sum())))
+                po.append(st["pops"] / max(1, int(reached.sum())))
+            key = f"vr{vr}_" + ("fifo" if delta == 0 else f"pq{delta}")
+            pq[key] = {"ms": statistics.median(ws), "edges_per_m_reached": statistics.mean(ed),
+                       "pops_per_reached": statistics.mean(po)}
+            if delta == 0:
+                out[f"bfs_rmat24_vr{vr}_ms"] = statistics.median(ws)
+                out[f"bfs_rmat24_vr{vr}_msgs_per_solve"] = st["msgs_sent"]
+            H.free()
+    out["priority_queue"] = pq
     gp = make_graph("rmat20_pr", dev)
     r_out = torch.empty(gp.n, dtype=torch.float64, device=dev)
     for vr in (1, 2, 8):

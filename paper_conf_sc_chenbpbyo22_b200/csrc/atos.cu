@@ -149,7 +149,7 @@ static bool valid_cfg(const atos_config &c) {
 // arena layout: identical computation on every rank
 // ---------------------------------------------------------------------------
 struct Layout {
-    size_t ctrl, depth, filt, hcb, rank, res, ring, ring2, in_hdr, in_pay, free_m, staging, parent, ghost, total;
+    size_t ctrl, depth, filt, hcb, vis, rank, res, ring, ring2, in_hdr, in_pay, free_m, staging, parent, ghost, total;
     uint64_t ring_cap;
     int64_t n_r;
 };
@@ -181,6 +181,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.depth = o;   o = al(o + (size_t)S.n * 4);
     L.filt = o;    o = al(o + (size_t)S.n);
     L.hcb = o;     o = al(o + (size_t)S.hub_chunks);
+    L.vis = o;     o = al(o + (S.pq && S.p == 1 ? ((size_t)S.n / 32 + 1) * 4 : 0));
     L.rank = o;    o = al(o + (size_t)L.n_r * 8);
     L.res = o;     o = al(o + (size_t)L.n_r * 8);
     L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
@@ -341,6 +342,7 @@ static RankDev build_view(const atos_graph *g, int lr) {
     d.depth = (uint32_t *)(b + L.depth);
     d.filt = (uint8_t *)(b + L.filt);
     d.hcb = (uint8_t *)(b + L.hcb);
+    d.vis = (g->S.pq && g->p == 1) ? (uint32_t *)(b + L.vis) : nullptr;
     d.pr_rank = (double *)(b + L.rank);
     d.pr_res = (double *)(b + L.res);
     d.pr_q = pr_q_of(L.n_r);
@@ -1028,6 +1030,10 @@ static KParams make_params(atos_graph *g) {
         kp.pq_th0 = (uint32_t)(g->cfg.pq_threshold > 0 ? g->cfg.pq_threshold : g->cfg.pq_delta);
         kp.keep = 0;
         kp.early = 0;
+        // buckets = levels on one rank: the visited bitmap replaces the depth words
+        // and the probe filter (atos_bfs1.cuh); ATOS_NO_VIS keeps them (A/B)
+        kp.vis = kp.bfs1 && kp.pq_delta == 1 && kp.pq_th0 == 1 && !ATOS_FILTER4 && !std::getenv("ATOS_NO_VIS");
+        if (kp.vis) kp.relax_red = 0;     // discoveries are decided by atomicOr with return: no fence before enqueue
     }
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
@@ -1044,9 +1050,10 @@ static bool l2_window(atos_graph *g, const KParams &kp, cudaAccessPolicyWindow &
     // keep the random-access state resident in L2 while the CSR column stream
     // passes through
     const LocalRank &me = g->loc[0];
-    void *base = APP == kApBfs ? (void *)(me.arena + (kp.filter ? me.L.filt : me.L.depth))
+    void *base = APP == kApBfs ? (void *)(me.arena + (kp.vis ? me.L.vis : kp.filter ? me.L.filt : me.L.depth))
                                : (void *)(me.arena + me.L.res);
-    size_t bytes = APP == kApBfs ? (size_t)g->n * (kp.filter ? 1 : 4) : (size_t)me.L.n_r * 8;
+    size_t bytes = APP == kApBfs ? (kp.vis ? ((size_t)g->n / 32 + 1) * 4 : (size_t)g->n * (kp.filter ? 1 : 4))
+                                 : (size_t)me.L.n_r * 8;
     bytes = std::min(bytes, g->window_max);
 #ifdef ATOS_CARVE_MAX   // experiment: the whole persisting limit as carve-out
     const size_t carve = g->persist_max;
@@ -1350,6 +1357,7 @@ extern "C" atos_status atos_pagerank(atos_graph *g, double alpha, double eps, do
     atos_status s = begin_solve(g, kp);
     if (s != ATOS_OK) return s;
     kp.pq = 0;                     // the priority queue orders BFS by depth only
+    kp.vis = 0;
     kp.alpha = alpha;
     kp.eps = eps;
     kp.eps_g = eps / (double)g->p;

@@ -39,6 +39,9 @@ __global__ void init_bfs_kernel(KParams kp) {
         }
         for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < kp.hub_chunks; i += (int64_t)gridDim.x * blockDim.x)
             R.hcb[i] = 255;     // hub bounds: unknown
+        if (kp.vis)             // visited bitmap: nothing visited
+            for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n / 32 + 1; i += (int64_t)gridDim.x * blockDim.x)
+                R.vis[i] = 0u;
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
 }
@@ -59,6 +62,7 @@ __global__ void seed_bfs_kernel(KParams kp, int64_t src) {
         if (src < R.v_begin || src >= R.v_end) continue;
         R.depth[src] = dw_make(0);
         filt_put_fresh(R.filt, src, 0u);
+        if (kp.vis) R.vis[src >> 5] |= 1u << (src & 31);
         const int q = kp.pq ? (int)(R.ctrl->pq_state.v & 1) : 0;   // the current bucket's ring
         const uint64_t idx = *q_tail(R, q);
         uint64_t *p = &q_slots(R, q)[idx & (R.ring_cap - 1)];
@@ -139,7 +143,11 @@ __global__ void gather_bfs_kernel(KParams kp, int32_t *out) {
         int o = 0;
         for (int k = 1; k < R.n_ranks; ++k) o += R.part[k] <= v ? 1 : 0;
         const int64_t nv = R.perm ? R.perm[v] : v;
-        const uint32_t d = dw_depth(__ldcg(R.peer_depth[o] + nv));
+        uint32_t d = dw_depth(__ldcg(R.peer_depth[o] + nv));
+        if (kp.vis) {            // visited-bitmap mode: depth bytes (the word only at depth >= 255)
+            const uint32_t b = __ldcg(R.filt + nv);
+            if (b < 255u) d = b;
+        }
         out[v] = d == kDepthInf ? -1 : (int32_t)d;
     }
 }

@@ -30,6 +30,19 @@
 //    filt(u) <= bound <= nd), so it is retired by one shared-memory byte load
 //    instead of a global probe.  Exactness is unchanged: only edges that
 //    cannot improve are skipped.
+//
+// 3. Visited bitmap (KParams::vis: the priority queue with threshold_delta 1,
+//    i.e. buckets = BFS levels).  A bucket only holds vertices of
+//    its level, and every vertex is discovered at its final depth (all vertices
+//    of smaller depth were expanded in earlier buckets), so the state a probe
+//    needs is ONE bit: visited or not.  The n-bit bitmap (8 MB at RMAT-26) stays
+//    in L2 -- the 67 MB byte filter did not (45 % L2 hit rate, 22 GB DRAM reads
+//    per RMAT-26 solve) -- and a stale L1 copy of a word only shows fewer bits,
+//    which costs an extra atomicOr, never a wrong result.  The discoverer is the
+//    one lane whose atomicOr set the bit: it stores the depth byte and enqueues,
+//    so there are no duplicate queue entries, no claim at pop, and no 4-byte
+//    depth words to read-modify-write in DRAM.  Hub bounds become "all 128 hubs
+//    of the chunk visited" (0) or unknown (255).
 #pragma once
 // (included inside namespace atos by atos_worker.cuh)
 
@@ -67,6 +80,20 @@ __device__ __forceinline__ void hub_refresh(Smem &s, const KParams &kp, int cta)
             // change nothing; stores into the array every worker copies from cost)
             if (lane == 0 && c < C && cm < hub_base(s)[c]) s.R.hcb[c] = (uint8_t)cm;
         }
+    }
+}
+
+// Visited-bitmap variant: chunk c (128 ids) = bitmap words 4c .. 4c+3; a warp
+// checks 8 chunks per load (lane l: word 4 * (c0 + l/4) + l%4).
+__device__ __forceinline__ void hub_refresh_vis(Smem &s, const KParams &kp, int cta) {
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t C = (uint32_t)kp.hub_n >> 7;
+    const uint32_t GW = (uint32_t)kp.ctas_per_rank * kWarps;
+    for (uint32_t cb = ((uint32_t)cta * kWarps + w) * 8u; cb < C; cb += GW * 8u) {
+        const uint32_t c = cb + (uint32_t)(lane >> 2);
+        const uint32_t x = c < C ? __ldcg(s.R.vis + 4 * (size_t)c + (lane & 3)) : 0u;
+        const uint32_t full = __ballot_sync(kFull, x == 0xFFFFFFFFu);
+        if ((lane & 3) == 0 && c < C && ((full >> lane) & 15u) == 15u && hub_base(s)[c] != 0) s.R.hcb[c] = 0;
     }
 }
 
@@ -139,6 +166,39 @@ __device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, con
     }
 }
 
+// Visited-bitmap relaxation of N edges per lane (all at candidate depth nd):
+// hub-bound test, bit probe (L1-cacheable: a stale word is conservative), and
+// for clear bits the atomicOr that decides the discoverer.  msk bit k = lane
+// discovered u[k] (store the depth byte, enqueue).
+template <int N>
+__device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                          uint32_t nd, uint32_t &msk, uint32_t &hits) {
+    uint32_t *const vis = s.R.vis;
+    const uint32_t H = (uint32_t)kp.hub_n;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        if ((uint32_t)u[k] < H && hcs[(uint32_t)u[k] >> 7] == 0) {
+            u[k] = -1;
+            ++hits;
+        }
+    }
+    uint32_t wd[N];
+#pragma unroll
+    for (int k = 0; k < N; ++k) wd[k] = u[k] >= 0 ? __ldca(vis + ((uint32_t)u[k] >> 5)) : 0xFFFFFFFFu;
+    msk = 0;
+#pragma unroll
+    for (int k = 0; k < N; ++k) {
+        const uint32_t bit = 1u << ((uint32_t)u[k] & 31u);
+        if (u[k] >= 0 && !(wd[k] & bit)) {
+            if (!(atomicOr(vis + ((uint32_t)u[k] >> 5), bit) & bit)) {
+                if (nd < 255u) stg_u8(s.R.filt + u[k], nd);
+                else s.R.depth[u[k]] = dw_make(nd);
+                msk |= 1u << k;
+            }
+        }
+    }
+}
+
 // largest li in [0, NL) with lq0[li] <= c (lq0[0] == 0 <= c)
 __device__ __forceinline__ uint32_t long_row_of(const BatchBuf &bb, uint32_t NL, uint32_t c) {
     uint32_t lo = 0, hi = NL - 1;
@@ -155,7 +215,7 @@ __device__ __forceinline__ uint32_t long_row_of(const BatchBuf &bb, uint32_t NL,
 // stream in flight (memory-level parallelism is what bounds the stream: a
 // warp's chunk is a dependent column -> probe -> relax chain).  A short chunk
 // is 128 edges of the packed short-row edge space.
-template <int G>
+template <int G, bool VIS>
 __device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KParams &kp, const int32_t *col,
                                            uint64_t pol, uint32_t NL, uint32_t c, uint32_t lane, const uint8_t *hcs,
                                            int64_t vb, uint32_t &wn, uint32_t &hits) {
@@ -181,16 +241,18 @@ __device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KP
 #pragma unroll
     for (int k = 0; k < 4 * G; ++k) nd[k] = r.nd;
     uint32_t msk;
-    relax_bfs1<4 * G>(s, kp, hcs, u, nd, msk, hits);
+    if constexpr (VIS) relax_vis<4 * G>(s, kp, hcs, u, r.nd, msk, hits);
+    else relax_bfs1<4 * G>(s, kp, hcs, u, nd, msk, hits);
     if (__any_sync(kFull, msk != 0)) {
         uint32_t item[4 * G];
         const uint32_t tag = r.nd >= s.pq_th ? kFarBit : 0u;     // priority queue (N1): far bucket
 #pragma unroll
         for (int k = 0; k < 4 * G; ++k) item[k] = (uint32_t)(u[k] - vb) | tag;
-        warp_append_mask<4 * G>(s, w, wn, msk, item, true);
+        warp_append_mask<4 * G>(s, w, wn, msk, item, kp.relax_red);
     }
 }
 
+template <bool VIS>
 __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t NL, uint32_t NLC, uint32_t ES,
                             uint32_t &wn) {
     const int w = threadIdx.x >> 5;
@@ -204,7 +266,7 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
     uint32_t hits = 0;
     for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
         if (c < NLC) {
-            long_chunk<kLongG>(s, bb, kp, col, pol, NL, c, lane, hcs, vb, wn, hits);
+            long_chunk<kLongG, VIS>(s, bb, kp, col, pol, NL, c, lane, hcs, vb, wn, hits);
             continue;
         }
         // short rows: packed edge space, coalesced 4-B column loads
@@ -224,12 +286,13 @@ __device__ void expand_bfs1(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t N
             }
         }
         uint32_t msk;
-        relax_bfs1<4>(s, kp, hcs, u, nd, msk, hits);
+        if constexpr (VIS) relax_vis<4>(s, kp, hcs, u, s.pq_th, msk, hits);     // one level per bucket
+        else relax_bfs1<4>(s, kp, hcs, u, nd, msk, hits);
         if (__any_sync(kFull, msk != 0)) {
             uint32_t item[4];
 #pragma unroll
             for (int k = 0; k < 4; ++k) item[k] = pq_tag((uint32_t)(u[k] - vb), nd[k], s.pq_th);
-            warp_append_mask<4>(s, w, wn, msk, item, true);
+            warp_append_mask<4>(s, w, wn, msk, item, kp.relax_red);
         }
     }
     if (kp.hub_n) {
@@ -262,19 +325,28 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
             const int64_t rb = ldg_i64_nc(R.row_ptr + v), re = ldg_i64_nc(R.row_ptr + v + 1);
             b = rb + (int64_t)pc * kp.split;
             deg = re - b < (int64_t)kp.split ? re - b : (int64_t)kp.split;
-            const uint32_t d = dw_depth(ld_relaxed_gpu_u32(R.depth + R.v_begin + v));
-            nd = d + 1;
-            if (d == kDepthInf || deg < 0) deg = 0;
+            if (kp.vis) {
+                nd = s.pq_th;              // buckets are levels: every item of this one has depth th - 1
+                if (deg < 0) deg = 0;
+            } else {
+                const uint32_t d = dw_depth(ld_relaxed_gpu_u32(R.depth + R.v_begin + v));
+                nd = d + 1;
+                if (d == kDepthInf || deg < 0) deg = 0;
+            }
         } else {
             const uint32_t v = it;
             b = ldg_i64_nc(R.row_ptr + v);
             deg = ldg_i64_nc(R.row_ptr + v + 1) - b;
-            // claim the expansion of v at its current depth; stale duplicates see
-            // the pending bit already cleared and are skipped
-            const uint32_t old = atom_and_u32(R.depth + R.v_begin + v, ~1u);
-            const uint32_t d = dw_depth(old);
-            nd = d + 1;
-            if (!(old & 1u) || d == kDepthInf) deg = 0;
+            if (kp.vis) {
+                nd = s.pq_th;              // enqueued once, by its discoverer, at its final depth th - 1
+            } else {
+                // claim the expansion of v at its current depth; stale duplicates see
+                // the pending bit already cleared and are skipped
+                const uint32_t old = atom_and_u32(R.depth + R.v_begin + v, ~1u);
+                const uint32_t d = dw_depth(old);
+                nd = d + 1;
+                if (!(old & 1u) || d == kDepthInf) deg = 0;
+            }
             if (kp.split > 0 && deg > 2 * (int64_t)kp.split && (int64_t)v < kPieceVMax &&
                 deg <= (int64_t)kp.split * kPieceMax) {
                 npc = (uint32_t)((deg - 1) / kp.split);   // pieces 1..npc go to the ring
@@ -345,10 +417,14 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     if (NLC + ES > 0) {
         const int w = tid >> 5;
         uint32_t wn = s.wn[w];
-        expand_bfs1(s, bb, kp, NL, NLC, ES, wn);
+        if (kp.vis) expand_bfs1<true>(s, bb, kp, NL, NLC, ES, wn);
+        else expand_bfs1<false>(s, bb, kp, NL, NLC, ES, wn);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }
-    if (hub && !(kp.hub_dbg & 1)) hub_refresh(s, kp, cta);
+    if (hub && !(kp.hub_dbg & 1)) {
+        if (kp.vis) hub_refresh_vis(s, kp, cta);
+        else hub_refresh(s, kp, cta);
+    }
 }
 

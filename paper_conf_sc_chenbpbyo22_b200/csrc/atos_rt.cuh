@@ -262,6 +262,7 @@ struct RankDev {
     uint32_t *depth;             // BFS: [n] global-indexed words dw (owned + ghost filter)
     uint8_t *filt;               // BFS: [n] probe filter, an upper bound of depth saturated at 255
     uint8_t *hcb;                // BFS hub bounds: [hub_chunks] upper bound of max filt over 128 hub ids
+    uint32_t *vis;               // BFS visited bitmap [n/32 + 1] (level-synchronous priority queue, KParams::vis)
     double *pr_rank;             // PR: [n_r], stored at pr_slot(local id)
     double *pr_res;              // PR: [n_r], stored at pr_slot(local id)
     double *pr_ghost;            // PR combining: [n] unsent residual for remote vertices, at pr_slot(global id, pr_q_of(n)); NULL = off
@@ -326,6 +327,8 @@ struct KParams {
     int32_t pq;              // BFS priority queue (N1): items of depth >= threshold go to the other ring
     uint32_t pq_th0;         // initial threshold (depths < pq_th0 form the first bucket)
     uint32_t pq_delta;       // threshold_delta: the threshold grows by this at every bucket advance
+    int32_t vis;             // single-rank BFS with pq_delta 1 (buckets = levels): visited bitmap instead
+                             // of depth words + probe filter (see atos_bfs1.cuh "visited bitmap")
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

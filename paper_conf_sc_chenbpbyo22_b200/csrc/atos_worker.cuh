@@ -275,7 +275,8 @@ __device__ __forceinline__ void ring_release(uint64_t *ring, uint64_t cap, uint6
 }
 
 // warp_flush_local with the priority queue (N1): far-tagged items go to the other ring.
-__device__ __noinline__ void warp_flush_local_pq(Smem &s, int w, uint32_t &wn, bool fence) {
+// (wn by value: a reference argument of a non-inlined call would live in local memory)
+__device__ __noinline__ void warp_flush_local_pq(Smem &s, int w, uint32_t wn, bool fence) {
     const uint32_t cnt = wn;
     const int lane = threadIdx.x & 31;
     const int q = s.pq_q;
@@ -314,6 +315,7 @@ __device__ void warp_flush_local(Smem &s, int w, uint32_t &wn, bool fence) {
     const int lane = threadIdx.x & 31;
     if (s.pq_th != kNoTh) {         // priority queue (N1): far-tagged items go to the other ring
         warp_flush_local_pq(s, w, wn, fence);
+        wn = 0;
         return;
     }
     unsigned long long base = 0;
@@ -439,9 +441,9 @@ __device__ bool warp_send_packet(Smem &s, const KParams &kp, int cta, int w, int
 
 // Whole warp: send full packets (and partial ones when `partial`) for every destination.
 template <int APP>
-__device__ __noinline__ void warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t &wn) {
+__device__ __noinline__ uint32_t warp_flush_remote(Smem &s, const KParams &kp, int cta, int w, bool batch_end, uint32_t wn) {
     const RankDev &R = s.R;
-    if (R.n_ranks <= 1) return;
+    if (R.n_ranks <= 1) return wn;
     const uint64_t now = globaltimer();
     for (int d = 0; d < R.n_ranks; ++d) {
         if (d == R.rank) continue;
@@ -457,9 +459,10 @@ __device__ __noinline__ void warp_flush_remote(Smem &s, const KParams &kp, int c
             go = __shfl_sync(kFull, go, 0);
             if (!go) break;
             const uint32_t cnt = pending < (uint32_t)kp.pkt ? pending : (uint32_t)kp.pkt;
-            if (!warp_send_packet<APP>(s, kp, cta, w, d, cnt, wn)) return;
+            if (!warp_send_packet<APP>(s, kp, cta, w, d, cnt, wn)) return wn;
         }
     }
+    return wn;
 }
 
 // Whole warp: lanes with pred stage a message (dst, v_local at dst, payload).
@@ -477,7 +480,7 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
         __syncwarp();
         if (s.wst[w][d] - s.wsh[w][d] + 32 > (uint32_t)kp.stage_cap) {
             // full packets out first (keeps room for this row)
-            warp_flush_remote<APP>(s, kp, cta, w, false, wn);
+            wn = warp_flush_remote<APP>(s, kp, cta, w, false, wn);
             __syncwarp();
         }
         const uint32_t t = s.wst[w][d];
@@ -496,7 +499,7 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
     }
     // aggregation off: the warp pushes what this 32-edge step produced right away
     // (Listing 5's per-warp remote push): packets of <= 32 messages
-    if (!kp.agg_on) warp_flush_remote<APP>(s, kp, cta, w, true, wn);
+    if (!kp.agg_on) wn = warp_flush_remote<APP>(s, kp, cta, w, true, wn);
 }
 
 // Whole warp: claim the ready prefix (up to kClaim packets) of one inbound
@@ -1342,7 +1345,7 @@ __device__ int batch_end(Smem &s, const KParams &kp, int cta, bool allow_keep) {
     __syncthreads();
     if constexpr (MULTI) {
         uint32_t wn = s.wn[w];
-        warp_flush_remote<APP>(s, kp, cta, w, true, wn);
+        wn = warp_flush_remote<APP>(s, kp, cta, w, true, wn);
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
         __syncthreads();
@@ -1459,7 +1462,19 @@ __device__ __noinline__ void pq_choose(Smem &s, const KParams &kp) {
             hi = lo + n;
         }
     }
-    if (lo != hi && slot_full_for(ld_relaxed_gpu(&q_slots(R, q)[lo & (R.ring_cap - 1)]), lo)) return;
+    if (lo != hi && slot_full_for(ld_relaxed_gpu(&q_slots(R, q)[lo & (R.ring_cap - 1)]), lo)) {
+        // The item may belong to a later bucket if ring q was swapped out since st
+        // was read (items still in a ring at a swap were all pushed after it: the
+        // ring was drained).  Re-read the state (the load is issued after the slot
+        // was seen full); if it moved, the batch goes back to its ring unexpanded.
+        if (ld_relaxed_gpu(&R.ctrl->pq_state.v) != st) s.pq_q = q ^ 1;
+        return;
+    }
+    // A reservation that overshot a ring's tail and is still open when the ring
+    // becomes the other bucket's (after a swap) receives that bucket's items.  They
+    // are popped (the reserved indices must be consumed) but not expanded -- their
+    // depth may not be final yet -- and go back to the end of that ring
+    // (pq_recycle), which also frees the worker's reservation.
     const int o = q ^ 1;
     const uint64_t lo2 = res_lo_q(s, o), hi2 = res_hi_q(s, o);
     if (lo2 != hi2 && slot_full_for(ld_relaxed_gpu(&q_slots(R, o)[lo2 & (R.ring_cap - 1)]), lo2)) {
@@ -1471,6 +1486,19 @@ __device__ __noinline__ void pq_choose(Smem &s, const KParams &kp) {
     const uint64_t t = ld_acquire_gpu(q_tail(R, q));
     if (f == t && ld_relaxed_gpu(q_tail(R, o)) > ld_relaxed_gpu(q_fin(R, o)))
         atomicCAS((unsigned long long *)&R.ctrl->pq_state.v, (unsigned long long)st, (unsigned long long)(st + 1));
+}
+
+// Priority queue: a batch popped from the NON-current ring (an old reservation,
+// see pq_choose) goes back to the end of that ring unexpanded.  Whole CTA.
+__device__ __noinline__ void pq_recycle(Smem &s, int B) {
+    const int tid = threadIdx.x, q = s.pop_q;
+    if (tid == 0) {
+        s.b64[0] = atomicAdd((unsigned long long *)q_tail(s.R, q), (unsigned long long)B);
+        s.c_pushes += (unsigned long long)B;
+    }
+    __syncthreads();
+    if (tid < B) ring_store(s.R, s.b64[0] + (uint64_t)tid, s.bb[0].v[tid], ring_base_q(s, q), q);
+    __syncthreads();
 }
 
 __device__ int pop_batch(Smem &s, const KParams &kp) {
@@ -1671,6 +1699,10 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
 #endif
             if (B > 0) {
                 const int B0 = B;
+                if (kp.pq && s.pop_q != s.pq_q) {      // not this bucket's: back to its ring
+                    pq_recycle(s, B);
+                    B = 0;
+                }
                 int chain = 0;
                 while (B > 0) {                 // work-keeping chain
                     if (tid == 0) s.c_pops += B;
@@ -1719,7 +1751,7 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         ++idle_streak;
         if constexpr (multi) {
             uint32_t wn = s.wn[w];
-            warp_flush_remote<APP>(s, kp, cta, w, true, wn);
+            wn = warp_flush_remote<APP>(s, kp, cta, w, true, wn);
             warp_flush_local(s, w, wn, false);
             if ((tid & 31) == 0) s.wn[w] = wn;
             report_staged(s, kp);

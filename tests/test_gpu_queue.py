@@ -52,7 +52,7 @@ def test_queue_tiny_ring_wraps_and_crosses_2_32(worker):
 
 
 def test_queue_push_only_fills_exactly():
-    threads, rounds = 1 << 12, 10
+    threads, rounds = 1 << 12, 16
     ms, _ = atos.queue_bench(32, "push", threads, rounds, ring_cap=threads * rounds, index_base=NEAR_2_32)
     assert ms > 0
 
