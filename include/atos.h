@@ -154,8 +154,10 @@ typedef struct {
                                  process (load/solve/free loops)               */
     int32_t pq_delta;         /* BFS priority queue (Listing 4's
                                  DistributedPriorityQueues threshold_delta,
-                                 P:629-639): 0 = FIFO queue (the
-                                 default); > 0 = every rank keeps two rings,
+                                 P:629-639): 0 = FIFO queue;
+                                 -1 = auto (the default): 1 on a skewed
+                                 single-rank graph of >= 2^25 vertices, else
+                                 FIFO; > 0 = every rank keeps two rings,
                                  the current bucket (candidate depth below the
                                  threshold) and the rest; workers pop only the
                                  current one, and when it is drained the rings

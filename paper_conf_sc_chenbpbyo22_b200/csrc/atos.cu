@@ -104,7 +104,7 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->pr_combine = 0;
     cfg->pool_retain = 0;
     cfg->pq_threshold = 0;
-    cfg->pq_delta = 0;
+    cfg->pq_delta = -1;
     return ATOS_OK;
 }
 
@@ -127,6 +127,18 @@ extern "C" atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *
     return ATOS_OK;
 }
 
+// Priority-queue layout (second ring, visited bitmap): pq_delta > 0, or the auto
+// choice (pq_delta = -1) on a single-rank graph of >= kPqAutoN vertices, where
+// the byte probe filter (n bytes) no longer stays in L2 and level buckets with
+// the n-bit visited bitmap win (RMAT-26 BFS 13.6 -> 10.2 ms; RMAT-24, whose
+// filter fits, 2.61 vs 2.78 ms FIFO).  Whether auto actually
+// orders by level is decided per solve from the degree skew (make_params).
+constexpr int64_t kPqAutoN = (int64_t)1 << 25;
+static int pq_layout(const atos_config &c, int64_t n) {
+    if (c.pq_delta > 0) return 1;
+    return c.pq_delta == -1 && c.n_ranks == 1 && c.virtual_ranks == 1 && n >= kPqAutoN ? 1 : 0;
+}
+
 static bool valid_cfg(const atos_config &c) {
     auto pow2 = [](int64_t x) { return x > 0 && (x & (x - 1)) == 0; };
     return c.worker_threads == kThreads && c.fetch_size >= 1 && c.fetch_size <= kThreads &&
@@ -142,7 +154,7 @@ static bool valid_cfg(const atos_config &c) {
             (c.split_edges >= 256 && c.split_edges <= (1 << 20) && pow2(c.split_edges))) &&
            (c.pr_combine == 0 || c.pr_combine == 1) && (c.pool_retain == 0 || c.pool_retain == 1) &&
            (c.discrete == 0 || (c.discrete == 1 && c.n_ranks == 1 && c.virtual_ranks == 1)) &&
-           c.pq_threshold >= 0 && c.pq_delta >= 0;
+           c.pq_threshold >= 0 && c.pq_delta >= -1;
 }
 
 // ---------------------------------------------------------------------------
@@ -555,7 +567,7 @@ extern "C" atos_status atos_arena_bytes(int64_t n, const int64_t *part, int32_t 
     else atos_partition_balanced(n, n_ranks, pt.data());
     Shape S{n, n_ranks, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs),
             148 * (cfg.ctas_per_sm ? cfg.ctas_per_sm : 2) / (cfg.virtual_ranks > 1 ? cfg.virtual_ranks : 1),
-            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
+            cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, pq_layout(cfg, n)};
     *bytes_out = make_layout(S, pt.data(), rank).total;
     return ATOS_OK;
 }
@@ -771,7 +783,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     } else {
         atos_partition_balanced(n, g->p, g->part.data());
     }
-    if (cfg.pq_delta > 0)      // priority queue items carry a bucket tag in bit 30
+    if (pq_layout(cfg, n))     // priority queue items carry a bucket tag in bit 30
         for (int r = 0; r < g->p; ++r)
             if (g->part[r + 1] - g->part[r] >= ((int64_t)1 << 30))
                 return fail(ATOS_ERR_INVALID_ARG, "priority queue: rank blocks must hold < 2^30 vertices");
@@ -818,7 +830,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     if (cpr < 1) return fail(ATOS_ERR_INVALID_ARG, "too many virtual ranks for the device");
     g->grid = cpr * g->n_local;
     g->S = Shape{n, g->p, cfg.channel_packets, cfg.agg_batch_msgs, stage_cap_for(cfg.agg_batch_msgs), cpr,
-                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, cfg.pq_delta > 0 ? 1 : 0};
+                 cfg.fetch_size, cfg.ring_cap_factor, cfg.pr_combine, 0, pq_layout(cfg, n)};
 
     if (cfg.stream) {
         g->stream = (cudaStream_t)cfg.stream;
@@ -833,7 +845,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
 
     LoadTrace tr;
     tr.mark(g->stream, "setup");
-    if ((cfg.relabel != 0 || cfg.keep_items < 0) && n > 1) {
+    if ((cfg.relabel != 0 || cfg.keep_items < 0 || (g->S.pq && cfg.pq_delta < 0)) && n > 1) {
         atos_status rs = compute_relabel(g, row_ptr, rp_dev);
         tr.mark(g->stream, "compute_relabel");
         if (rs != ATOS_OK) return rs;
@@ -1022,12 +1034,16 @@ static KParams make_params(atos_graph *g) {
     kp.static_chunks = std::getenv("ATOS_DYNAMIC_CHUNKS") ? 0 : 1;
     if (const char *f = std::getenv("ATOS_TEST_FAULT"))   // test-only fault injection (T6 error paths)
         kp.fault = std::strcmp(f, "capacity") == 0 ? kFaultCapacity : std::strcmp(f, "timeout") == 0 ? kFaultTimeout : 0;
-    if (g->S.pq) {
+    if (g->S.pq && (g->cfg.pq_delta > 0 || g->skewed)) {
         // priority queue (N1): no work keeping (a kept chain would bypass the
-        // buckets) and no early reservation (it is ring-0 only)
+        // buckets) and no early reservation (it is ring-0 only).  Auto
+        // (pq_delta = -1, large single-rank graphs): level buckets on skewed
+        // graphs; a non-skewed (high-diameter) graph keeps the FIFO queue and
+        // work keeping, one bucket per level would serialise its ~10^4 levels
+        const uint32_t delta = g->cfg.pq_delta > 0 ? (uint32_t)g->cfg.pq_delta : 1u;
         kp.pq = 1;
-        kp.pq_delta = (uint32_t)g->cfg.pq_delta;
-        kp.pq_th0 = (uint32_t)(g->cfg.pq_threshold > 0 ? g->cfg.pq_threshold : g->cfg.pq_delta);
+        kp.pq_delta = delta;
+        kp.pq_th0 = g->cfg.pq_threshold > 0 ? (uint32_t)g->cfg.pq_threshold : delta;
         kp.keep = 0;
         kp.early = 0;
         // buckets = levels on one rank: the visited bitmap replaces the depth words

@@ -108,12 +108,13 @@ def test_relabel_and_hub_cache_config_validation():
     cfg = atos.default_config()
     assert cfg.relabel == 2 and cfg.hub_cache == -1          # auto / auto
     assert cfg.split_edges == -1 and cfg.keep_items == -1     # auto
+    assert cfg.pq_delta == -1                                  # auto (N1 level buckets on large skewed graphs)
     rp = np.array([0, 1, 1], dtype=np.int64)
     col = np.array([1], dtype=np.int32)
     for bad in (dict(relabel=3), dict(hub_cache=33), dict(hub_cache=1 << 23), dict(hub_cache=-2),
                 dict(hub_cache=32, virtual_ranks=2), dict(hub_cache=200), dict(split_edges=100), dict(split_edges=128),
                 dict(split_edges=1 << 21), dict(split_edges=-2), dict(pr_combine=2), dict(keep_items=-2), dict(keep_mode=2), dict(discrete=2),
-                dict(discrete=1, virtual_ranks=2), dict(discrete=1, n_ranks=2), dict(pq_delta=-1), dict(pq_threshold=-1)):
+                dict(discrete=1, virtual_ranks=2), dict(discrete=1, n_ranks=2), dict(pq_delta=-2), dict(pq_threshold=-1)):
         with pytest.raises(atos.AtosError) as e:
             atos.Graph(rp, col, **bad)
         assert e.value.status == 1, bad
