@@ -61,7 +61,9 @@ def arm_config(args, g, srcs, world):
             "sources": len(srcs), "partition": "1d-balanced", "parallelism": f"vertex-1d x{world}",
             "aggregation": bool(args.agg),
             "vertex_order": "degree-relabeled inside rank blocks (atos_config.relabel=auto); outputs in generator ids",
-            "probe": "u8 depth-bound filter on skewed graphs (atos_config.probe_filter=auto)",
+            "queue": ("one rank: level buckets (N1 priority queue, threshold_delta 1; atos_config.pq_delta=auto) "
+                      "with an n-bit visited bitmap and claim at pop; several ranks: FIFO queue with the "
+                      "u8 depth-bound filter (atos_config.probe_filter=auto)"),
             "l2": ("no flush: CSR inputs larger than L2 (%.2f GB > 126 MB)" % ((g.nnz * 4 + g.n * 8) / 1e9))
             if g.nnz * 4 + g.n * 8 > 126e6 else "CSR fits L2 (%.1f MB): a latency figure, not a bandwidth one"
                                                 % ((g.nnz * 4 + g.n * 8) / 1e6)}
@@ -535,11 +537,13 @@ def cpu_baseline_pr():
     gp = inputs.make_config("rmat20_pr")
     rp, col = gp.numpy()
     out = {"graph": gp.name, "tol": 1e-12}
-    for name, nt in (("one_core", 1), ("all_cores", 0)):
+    # all cores: an explicit thread count (OMP_NUM_THREADS may be 1 in the environment;
+    # the r2 box reported omp_get_max_threads() == 1 with 16 cores)
+    ncores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+    for name, nt in (("one_core", 1), ("all_cores", ncores)):
         t0 = time.perf_counter()
         _, it, delta = oracle.pagerank(rp, col, 0.85, 1e-12, nthreads=nt)
-        out[name] = {"seconds": time.perf_counter() - t0, "iterations": it,
-                     "threads": 1 if nt == 1 else oracle.max_threads()}
+        out[name] = {"seconds": time.perf_counter() - t0, "iterations": it, "threads": nt}
     out["nproc"] = os.cpu_count()
     try:
         out["cpu_model"] = next(l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name"))

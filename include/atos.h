@@ -156,7 +156,7 @@ typedef struct {
                                  DistributedPriorityQueues threshold_delta,
                                  P:629-639, P:1350-1359): 0 = FIFO queue;
                                  -1 = auto (the default): 1 on a skewed
-                                 single-rank graph of >= 2^25 vertices, else
+                                 single-rank graph of >= 2^20 vertices, else
                                  FIFO; > 0 = every rank keeps two rings,
                                  the current bucket (candidate depth below the
                                  threshold) and the rest; workers pop only the

@@ -127,13 +127,15 @@ extern "C" atos_status atos_validate_csr(const int64_t *row_ptr, const int32_t *
     return ATOS_OK;
 }
 
-// Priority-queue layout (second ring, visited bitmap): pq_delta > 0, or the auto
-// choice (pq_delta = -1) on a single-rank graph of >= kPqAutoN vertices, where
-// the byte probe filter (n bytes) no longer stays in L2 and level buckets with
-// the n-bit visited bitmap win (RMAT-26 BFS 13.6 -> 10.2 ms; RMAT-24, whose
-// filter fits, 2.61 vs 2.78 ms FIFO).  Whether auto actually
-// orders by level is decided per solve from the degree skew (make_params).
-constexpr int64_t kPqAutoN = (int64_t)1 << 25;
+// Priority-queue layout (second ring, visited + claim bitmaps): pq_delta > 0, or
+// the auto choice (pq_delta = -1) on a single-rank graph of >= kPqAutoN
+// vertices, where level buckets with the n-bit visited bitmap and claim at pop
+// win over the FIFO queue with the byte filter (FIFO -> buckets, ms: RMAT-26
+// 13.5 -> 8.62, RMAT-24 2.57 -> 2.42, RMAT-22 0.85 -> 0.81, RMAT-20 0.58 ->
+// 0.41; RMAT-18 0.26 vs 0.27 and RMAT-16 0.14 vs 0.18 lose).
+// Whether auto actually orders by level is decided per solve from the degree
+// skew (make_params).
+constexpr int64_t kPqAutoN = (int64_t)1 << 20;
 static int pq_layout(const atos_config &c, int64_t n) {
     if (c.pq_delta > 0) return 1;
     return c.pq_delta == -1 && c.n_ranks == 1 && c.virtual_ranks == 1 && n >= kPqAutoN ? 1 : 0;
@@ -193,7 +195,7 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
     L.depth = o;   o = al(o + (size_t)S.n * 4);
     L.filt = o;    o = al(o + (size_t)S.n);
     L.hcb = o;     o = al(o + (size_t)S.hub_chunks);
-    L.vis = o;     o = al(o + (S.pq && S.p == 1 ? ((size_t)S.n / 32 + 1) * 4 : 0));
+    L.vis = o;     o = al(o + (S.pq && S.p == 1 ? ((size_t)S.n / 32 + 1) * 8 : 0));   // visited + claimed bitmaps
     L.rank = o;    o = al(o + (size_t)L.n_r * 8);
     L.res = o;     o = al(o + (size_t)L.n_r * 8);
     L.ring = o;    o = al(o + (size_t)L.ring_cap * 8);
@@ -1050,6 +1052,9 @@ static KParams make_params(atos_graph *g) {
         // and the probe filter (atos_bfs1.cuh); ATOS_NO_VIS keeps them (A/B)
         kp.vis = kp.bfs1 && kp.pq_delta == 1 && kp.pq_th0 == 1 && !ATOS_FILTER4 && !std::getenv("ATOS_NO_VIS");
         if (kp.vis) kp.relax_red = 0;     // discoveries are decided by atomicOr with return: no fence before enqueue
+        // claim at pop (RED discoveries, one atomicOr per pop): RMAT-26 9.81 -> 8.62 ms,
+        // RMAT-24 2.72 -> 2.43 ms; ATOS_VIS_NOCLAIM restores the discoverer's atomicOr (A/B)
+        if (kp.vis && !std::getenv("ATOS_VIS_NOCLAIM")) kp.vis_claim = 1;
     }
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;
@@ -1068,7 +1073,7 @@ static bool l2_window(atos_graph *g, const KParams &kp, cudaAccessPolicyWindow &
     const LocalRank &me = g->loc[0];
     void *base = APP == kApBfs ? (void *)(me.arena + (kp.vis ? me.L.vis : kp.filter ? me.L.filt : me.L.depth))
                                : (void *)(me.arena + me.L.res);
-    size_t bytes = APP == kApBfs ? (kp.vis ? ((size_t)g->n / 32 + 1) * 4 : (size_t)g->n * (kp.filter ? 1 : 4))
+    size_t bytes = APP == kApBfs ? (kp.vis ? ((size_t)g->n / 32 + 1) * (kp.vis_claim ? 8 : 4) : (size_t)g->n * (kp.filter ? 1 : 4))
                                  : (size_t)me.L.n_r * 8;
     bytes = std::min(bytes, g->window_max);
 #ifdef ATOS_CARVE_MAX   // experiment: the whole persisting limit as carve-out

@@ -40,8 +40,8 @@ __global__ void init_bfs_kernel(KParams kp) {
         for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < kp.hub_chunks; i += (int64_t)gridDim.x * blockDim.x)
             R.hcb[i] = 255;     // hub bounds: unknown
         if (kp.vis)             // visited bitmap: nothing visited
-            for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n / 32 + 1; i += (int64_t)gridDim.x * blockDim.x)
-                R.vis[i] = 0u;
+            for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 2 * (n / 32 + 1); i += (int64_t)gridDim.x * blockDim.x)
+                R.vis[i] = 0u;  // (and the claim bitmap behind it)
         if (blockIdx.x == 0 && threadIdx.x == 0) R.ctrl->error.v = 0;
     }
 }

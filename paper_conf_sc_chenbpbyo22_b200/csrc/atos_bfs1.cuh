@@ -189,6 +189,21 @@ __device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, cons
     uint32_t wd[N];
 #pragma unroll
     for (int k = 0; k < N; ++k) wd[k] = u[k] >= 0 ? __ldca(vis + ((uint32_t)u[k] >> 5)) : 0xFFFFFFFFu;
+    if (kp.vis_claim) {
+        // claim at pop: the bit is only a filter, set fire-and-forget (RED); a
+        // vertex two lanes (or a stale probe) both see clear is enqueued twice and
+        // the second pop loses the claim
+        msk = 0;
+#pragma unroll
+        for (int k = 0; k < N; ++k) {
+            const uint32_t bit = 1u << ((uint32_t)u[k] & 31u);
+            if (u[k] >= 0 && !(wd[k] & bit)) {
+                atomicOr(vis + ((uint32_t)u[k] >> 5), bit);
+                msk |= 1u << k;
+            }
+        }
+        return;
+    }
     // all of the lane's atomics are issued before the first result is used (the
     // depth stores below would otherwise order each atomic after the previous
     // one's round trip: the compiler cannot tell the byte array from the bitmap)
@@ -360,6 +375,20 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
             deg = ldg_i64_nc(R.row_ptr + v + 1) - b;
             if (kp.vis) {
                 nd = s.pq_th;              // enqueued once, by its discoverer, at its final depth th - 1
+                if (kp.vis_claim) {
+                    // claim at pop: the first pop of v (in its own level's bucket) wins
+                    // and stores v's depth; duplicates are skipped
+                    const uint64_t gv = (uint64_t)(R.v_begin + v);
+                    const uint32_t bit = 1u << (gv & 31u);
+                    uint32_t *const claim = R.vis + ((uint64_t)R.n >> 5) + 1;
+                    if (atomicOr(claim + (gv >> 5), bit) & bit) {
+                        deg = 0;
+                    } else if (nd - 1 < 255u) {
+                        stg_u8(R.filt + gv, nd - 1);
+                    } else {
+                        R.depth[gv] = dw_make(nd - 1);
+                    }
+                }
             } else {
                 // claim the expansion of v at its current depth; stale duplicates see
                 // the pending bit already cleared and are skipped

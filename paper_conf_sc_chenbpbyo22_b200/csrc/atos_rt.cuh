@@ -329,6 +329,8 @@ struct KParams {
     uint32_t pq_delta;       // threshold_delta: the threshold grows by this at every bucket advance
     int32_t vis;             // single-rank BFS with pq_delta 1 (buckets = levels): visited bitmap instead
                              // of depth words + probe filter (see atos_bfs1.cuh "visited bitmap")
+    int32_t vis_claim;       // with vis: discoveries are fire-and-forget red.or, the expansion is claimed
+                             // at pop in a second bitmap (atos_bfs1.cuh "claim at pop")
     int64_t agg_age_ns;
     int64_t watchdog_ns;
     uint64_t epoch;

@@ -54,7 +54,12 @@ def main():
         g = inputs.csr_from_edges(n, idx, idx + 1, symmetrize=True)
         srcs = [0]
     else:
-        g = inputs.make_config(args.graph, device="cuda")
+        import re
+        m = re.fullmatch(r"rmat(\d+)", args.graph)
+        if m and args.graph not in inputs.CONFIGS:      # any RMAT scale, configs[2]'s recipe
+            g = inputs.make_config("rmat24", device="cuda", scale=int(m.group(1)))
+        else:
+            g = inputs.make_config(args.graph, device="cuda")
         srcs = [0] if args.graph in ("kron12", "grid4900") else inputs.bfs_sources(g, 8)
     print(f"graph {g.name} n={g.n} nnz={g.nnz} gen {time.time()-t0:.1f}s", flush=True)
     for cfg in json.loads(args.configs):

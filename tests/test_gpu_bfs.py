@@ -186,13 +186,15 @@ def test_rmat24_config2_full_size_virtual_ranks(vr):
 
 
 @pytest.mark.slow
-def test_rmat24_config2_full_size():
-    """BASELINE configs[2] at full size, the launch configuration bench.py times."""
+@pytest.mark.parametrize("pq", [-1, 0])
+def test_rmat24_config2_full_size(pq):
+    """BASELINE configs[2] at full size: the launch configuration bench.py times
+    (auto: level buckets) and the FIFO queue with the byte filter."""
     g = inputs.make_config("rmat24", device="cuda")
     rp, col = g.row_ptr, g.col
     srcs = inputs.bfs_sources(g, 2)
     rpn, coln = g.numpy()
-    with atos.Graph(rp, col) as G:
+    with atos.Graph(rp, col, pq_delta=pq) as G:
         for s in srcs:
             d = G.bfs(s)
             want = oracle.bfs(rpn, coln, s)
@@ -359,7 +361,9 @@ def test_rmat26_north_star_full_size():
         G.bfs(srcs[1], depth_out=depth)
         G.sync()
         assert bfs_properties_hold(g.row_ptr, g.col, depth, srcs[1])
-        d0 = G.bfs(srcs[0])
+        d0, st = G.bfs(srcs[0], stats=True)
+    # the default (pq_delta = -1, auto) orders this graph by level buckets (N1)
+    assert st["pq_buckets"] > 0
     rpn, coln = g.numpy()
     assert np.array_equal(d0, oracle.bfs(rpn, coln, srcs[0]))
 

@@ -129,3 +129,26 @@ def test_pq_rmat24_config2_full_size():
     want = oracle.bfs(rp, col, src)
     assert np.array_equal(d, want)
     assert st["edges"] == m_reached(rp, d)
+
+
+@pytest.mark.parametrize("var", ["ATOS_VIS_NOCLAIM", "ATOS_NO_VIS"])
+def test_pq_delta1_switches(monkeypatch, var):
+    # the level-bucket variants behind the A/B switches: discoverer
+    # atomicOr instead of claim at pop; depth words + filter instead of the bitmap
+    monkeypatch.setenv(var, "1")
+    for g, src in ((inputs.rmat(15, 16, 2, symmetric=True), None), (inputs.road_grid(80, 60, 3), 0)):
+        rp, col = g.numpy()
+        s = inputs.bfs_sources(g, 1, seed=5)[0] if src is None else src
+        d, st = run_pq(rp, col, s, pq_delta=1)
+        assert st["pq_buckets"] == d.max()
+
+
+def test_pq_auto_is_fifo_on_small_graphs():
+    # auto (the default) keeps the FIFO queue below 2^20 vertices and on non-skewed graphs
+    g = inputs.rmat(14, 16, 1, symmetric=True)
+    rp, col = g.numpy()
+    src = inputs.bfs_sources(g, 1)[0]
+    with atos.Graph(rp, col) as G:
+        d, st = G.bfs(src, stats=True)
+    assert np.array_equal(d, oracle.bfs(rp, col, src))
+    assert st["pq_buckets"] == 0 and st["far_pushes"] == 0
