@@ -531,17 +531,17 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
         dfree(g, g->loc[lr].row_ptr);
         dfree(g, g->loc[lr].col);
     }
-    cudaFree(g->d_ranks);
+    dfree(g, g->d_ranks);
     dfree(g, g->d_depth_full);
     dfree(g, g->d_perm);
     dfree(g, g->d_inv);
-    cudaFree(g->d_accs);
+    dfree(g, g->d_accs);
     if (g->stream) cudaStreamSynchronize(g->stream);
     for (int a = 0; a < 2; ++a) {
         if (g->dexec[a]) cudaGraphExecDestroy(g->dexec[a]);
         if (g->dgraph[a]) cudaGraphDestroy(g->dgraph[a]);
     }
-    cudaFree(g->d_kp);
+    if (g->d_kp) cudaFree(g->d_kp);
     if (g->ev_begin) cudaEventDestroy(g->ev_begin);
     if (g->ev_w0) cudaEventDestroy(g->ev_w0);
     if (g->ev_w1) cudaEventDestroy(g->ev_w1);
@@ -733,10 +733,10 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
     const cudaError_t e = cudaStreamSynchronize(st);
     cudaStreamSynchronize(cs);
     for (size_t i = 0; i + 3 < tev.size(); i += 4) {
-        float a = 0, b2 = 0;
-        cudaEventElapsedTime(&a, tev[i], tev[i + 1]);
-        cudaEventElapsedTime(&b2, tev[i + 2], tev[i + 3]);
-        fprintf(stderr, "[atos load]   chunk %zu: copy %.2f ms, permute %.2f ms\n", i / 4, a, b2);
+        float t[4] = {0, 0, 0, 0};
+        for (int j = 0; j < 4; ++j) cudaEventElapsedTime(&t[j], tev[0], tev[i + j]);
+        fprintf(stderr, "[atos load]   chunk %zu: copy %.2f ms, permute %.2f ms (copy %.2f-%.2f, permute %.2f-%.2f ms)\n",
+                i / 4, t[1] - t[0], t[3] - t[2], t[0], t[1], t[2], t[3]);
     }
     for (cudaEvent_t x : tev) cudaEventDestroy(x);
     for (int k = 0; k < 2; ++k) { cudaEventDestroy(ev_in[k]); cudaEventDestroy(ev_out[k]); }
@@ -860,7 +860,7 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         g->S.hub_chunks = g->hub_chunks;
     }
     unsigned long long *d_bad = nullptr;
-    CU(cudaMalloc(&d_bad, sizeof(unsigned long long)));
+    CU(dmalloc(g, &d_bad, sizeof(unsigned long long)));   // (stream-ordered: cudaMalloc/cudaFree synchronise the device)
     CU(cudaMemsetAsync(d_bad, 0, sizeof(unsigned long long), g->stream));
     for (int lr = 0; lr < g->n_local; ++lr) {
         LocalRank &me = g->loc[lr];
@@ -890,17 +890,17 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
             unsigned long long bad0 = 0;
             CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
             CU(cudaStreamSynchronize(g->stream));
-            if (bad0) { cudaFree(d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone"); }
+            if (bad0) { dfree(g, d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone"); }
             atos_status rs = relabel_rows_streamed(g, me, row_ptr, col, d_bad);
-            if (rs != ATOS_OK) { cudaFree(d_bad); return rs; }
+            if (rs != ATOS_OK) { dfree(g, d_bad); return rs; }
             tr.mark(g->stream, "relabel rows (streamed)");
         } else if (g->d_perm) {   // rows must be valid before they are permuted
             unsigned long long bad0 = 0;
             CU(cudaMemcpyAsync(&bad0, d_bad, sizeof(bad0), cudaMemcpyDeviceToHost, g->stream));
             CU(cudaStreamSynchronize(g->stream));
-            if (bad0) { cudaFree(d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: invalid row_ptr or column index"); }
+            if (bad0) { dfree(g, d_bad); return fail(ATOS_ERR_INVALID_ARG, "csr: invalid row_ptr or column index"); }
             atos_status rs = relabel_rows(g, me);
-            if (rs != ATOS_OK) { cudaFree(d_bad); return rs; }
+            if (rs != ATOS_OK) { dfree(g, d_bad); return rs; }
             tr.mark(g->stream, "relabel rows");
         }
         const uint64_t nfree = g->p > 1 ? (uint64_t)g->p * g->S.cp : 0;
@@ -928,13 +928,13 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
     unsigned long long bad = 0;
     CU(cudaMemcpyAsync(&bad, d_bad, sizeof(bad), cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
-    cudaFree(d_bad);
+    dfree(g, d_bad);
     if (bad & 1) return fail(ATOS_ERR_INVALID_ARG, "csr: row_ptr not monotone");
     if (bad & 2) return fail(ATOS_ERR_INVALID_ARG, "csr: column index out of [0, n)");
 
-    CU(cudaMalloc(&g->d_ranks, sizeof(RankDev) * g->n_local));
+    CU(dmalloc(g, &g->d_ranks, sizeof(RankDev) * g->n_local));
     CU(dmalloc(g, &g->d_depth_full, (size_t)n * 4));
-    CU(cudaMalloc(&g->d_accs, sizeof(int64_t *) * kMaxRanks));
+    CU(dmalloc(g, &g->d_accs, sizeof(int64_t *) * kMaxRanks));
     g->connected = !g->multiproc;
     for (int lr = 0; lr < g->n_local; ++lr)    // the 16-B column loads of atos_bfs1.cuh need this
         if (((uintptr_t)g->loc[lr].col & 15) != 0)

@@ -133,13 +133,16 @@ __device__ __forceinline__ void hub_fill_unknown(Smem &s, const KParams &kp) {  
     for (int i = threadIdx.x; i < kp.hub_chunks; i += kThreads) hub_base(s)[i] = 255;
 }
 
-// Relax N edges per lane (u[k] < 0: no edge): hub-bound test, filter probe,
-// red.min + filter store on the probe's verdict (relax_red; duplicates are
-// skipped at pop by the pending bit, the flush fences before publishing).
+// Relaxation of N edges per lane in two phases, probe_* (hub-bound test, issue
+// the probe loads) and finish_* (decide, relax), so that a pipelined expansion
+// (ATOS_CHUNK_PIPE) can put the next chunk's column loads between them.
+//
+// Filter mode (u[k] < 0: no edge): hub-bound test, filter probe, red.min +
+// filter store on the probe's verdict (relax_red; duplicates are skipped at pop
+// by the pending bit, the flush fences before publishing).
 template <int N>
-__device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
-                                           const uint32_t (&nd)[N], uint32_t &msk, uint32_t &hits) {
-    uint32_t *const depth = s.R.depth;
+__device__ __forceinline__ void probe_bfs1(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                           const uint32_t (&nd)[N], uint32_t (&f)[N], uint32_t &hits) {
     uint8_t *const filt = s.R.filt;
     const uint32_t H = (kp.hub_dbg & 4) ? 0u : (uint32_t)kp.hub_n;
     uint32_t hm = 0;                  // slots retired by the hub bound (statistics: one popc)
@@ -154,9 +157,15 @@ __device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, con
         }
     }
     hits += __popc(hm);
-    uint32_t f[N];
 #pragma unroll
     for (int k = 0; k < N; ++k) f[k] = u[k] >= 0 ? ldg_u8(filt + u[k]) : 0u;
+}
+
+template <int N>
+__device__ __forceinline__ void finish_bfs1(const Smem &s, const int32_t (&u)[N], const uint32_t (&nd)[N],
+                                            const uint32_t (&f)[N], uint32_t &msk) {
+    uint32_t *const depth = s.R.depth;
+    uint8_t *const filt = s.R.filt;
     msk = 0;
 #pragma unroll
     for (int k = 0; k < N; ++k) {
@@ -168,15 +177,23 @@ __device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, con
     }
 }
 
-// Visited-bitmap relaxation of N edges per lane (all at candidate depth nd):
-// hub-bound test, bit probe (L1-cacheable: a stale word is conservative), and
-// for clear bits the atomicOr that decides the discoverer.  msk bit k = lane
-// discovered u[k] (store the depth byte, enqueue).
 template <int N>
-__device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
-                                          uint32_t nd, uint32_t &msk, uint32_t &hits) {
+__device__ __forceinline__ void relax_bfs1(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                           const uint32_t (&nd)[N], uint32_t &msk, uint32_t &hits) {
+    uint32_t f[N];
+    probe_bfs1<N>(s, kp, hcs, u, nd, f, hits);
+    finish_bfs1<N>(s, u, nd, f, msk);
+}
+
+// Visited-bitmap mode (all N edges at candidate depth nd): hub-bound test, bit
+// probe (L1-cacheable: a stale word is conservative), then for clear bits
+// either a fire-and-forget RED.OR (claim at pop, the default) or the
+// atomicOr-with-return that decides the discoverer.  msk bit k = enqueue u[k].
+template <int N>
+__device__ __forceinline__ void probe_vis(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                          uint32_t (&wd)[N], uint32_t &hits) {
     uint32_t *const vis = s.R.vis;
-    const uint32_t H = (uint32_t)kp.hub_n;
+    const uint32_t H = (kp.hub_dbg & 4) ? 0u : (uint32_t)kp.hub_n;
     uint32_t hm = 0;
 #pragma unroll
     for (int k = 0; k < N; ++k) {
@@ -186,9 +203,14 @@ __device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, cons
         }
     }
     hits += __popc(hm);
-    uint32_t wd[N];
 #pragma unroll
     for (int k = 0; k < N; ++k) wd[k] = u[k] >= 0 ? __ldca(vis + ((uint32_t)u[k] >> 5)) : 0xFFFFFFFFu;
+}
+
+template <int N>
+__device__ __forceinline__ void finish_vis(const Smem &s, const KParams &kp, const int32_t (&u)[N], uint32_t nd,
+                                           const uint32_t (&wd)[N], uint32_t &msk) {
+    uint32_t *const vis = s.R.vis;
     if (kp.vis_claim) {
         // claim at pop: the bit is only a filter, set fire-and-forget (RED); a
         // vertex two lanes (or a stale probe) both see clear is enqueued twice and
@@ -226,6 +248,14 @@ __device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, cons
             msk |= 1u << k;
         }
     }
+}
+
+template <int N>
+__device__ __forceinline__ void relax_vis(const Smem &s, const KParams &kp, const uint8_t *hcs, int32_t (&u)[N],
+                                          uint32_t nd, uint32_t &msk, uint32_t &hits) {
+    uint32_t wd[N];
+    probe_vis<N>(s, kp, hcs, u, wd, hits);
+    finish_vis<N>(s, kp, u, nd, wd, msk);
 }
 
 // Largest li in [0, NL) with lq0[li] <= c, searched forward from li0 (a row
@@ -285,6 +315,99 @@ __device__ __forceinline__ void long_chunk(Smem &s, const BatchBuf &bb, const KP
 #pragma unroll
         for (int k = 0; k < 4 * G; ++k) item[k] = (uint32_t)(u[k] - vb) | tag;
         warp_append_mask<4 * G>(s, w, wn, msk, item, kp.relax_red);
+    }
+}
+
+#ifndef ATOS_CHUNK_PIPE
+#define ATOS_CHUNK_PIPE 1     // 1 = next chunk's columns issued before this chunk's probes (default), 2 = after, 0 = off (A/B)
+#endif
+
+// One chunk's column ids in flight (pipelined expansion, ATOS_CHUNK_PIPE).
+struct ChunkFetch {
+    int32_t u[4];       // raw column ids (long chunk: valid where vm says so; short: -1 = no edge)
+    uint32_t nd[4];     // candidate depth per slot
+    uint32_t vm;        // valid-slot mask of a long chunk (0xF for short chunks)
+};
+
+__device__ __forceinline__ void fetch_chunk(const BatchBuf &bb, const int32_t *col, uint64_t pol, uint32_t NL,
+                                            uint32_t NLC, uint32_t ES, uint32_t c, uint32_t lane, uint32_t below,
+                                            uint32_t &lcur, ChunkFetch &f) {
+    if (c < NLC) {
+        const uint32_t li = c < (uint32_t)kLcv ? bb.lcv[c] : long_row_from(bb, NL, c, lcur, lane);
+        lcur = li;
+        const BRec r = bb.rec[kThreads - 1 - li];
+        const uint32_t lo = (uint32_t)(r.base & 3);
+        const int64_t a = r.base - lo;
+        const uint32_t rel = (c - bb.lq0[li]) * (uint32_t)kCh1 + 4u * lane;
+        const uint32_t end = lo + r.len;
+        f.vm = (uint32_t)(rel >= lo && rel < end) | ((uint32_t)(rel + 1 >= lo && rel + 1 < end) << 1) |
+               ((uint32_t)(rel + 2 >= lo && rel + 2 < end) << 2) | ((uint32_t)(rel + 3 < end) << 3);
+        if (rel < end) {
+            const int4 v = ld_stream4(col + a + rel, pol);
+            f.u[0] = v.x; f.u[1] = v.y; f.u[2] = v.z; f.u[3] = v.w;
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) f.nd[k] = r.nd;
+        return;
+    }
+    const uint32_t c0 = (c - NLC) * (uint32_t)kCh1;
+    f.vm = 0xFu;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint32_t e = c0 + 32u * k + lane;
+        f.u[k] = -1;
+        f.nd[k] = 0;
+        if (e < ES) {
+            const uint32_t wd = e >> 5;
+            const BRec r = bb.rec[bb.rowmap[wd] + __popc(bb.bm[wd] & below)];
+            f.u[k] = ld_stream(col + r.base + e, pol);
+            f.nd[k] = r.nd;
+        }
+    }
+}
+
+template <bool VIS>
+__device__ void expand_bfs1_pipe(Smem &s, BatchBuf &bb, const KParams &kp, uint32_t NL, uint32_t NLC, uint32_t ES,
+                                 uint32_t &wn) {
+    const int w = threadIdx.x >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    const int32_t *const col = s.R.col;
+    const uint8_t *const hcs = hub_base(s);
+    const uint64_t pol = policy_evict_first();
+    const uint32_t below = lane == 31 ? 0xFFFFFFFEu : (((2u << lane) - 1u) & ~1u);
+    const uint32_t ntot = NLC + (ES + kCh1 - 1) / kCh1;
+    const int64_t vb = s.R.v_begin;
+    uint32_t hits = 0, lcur = 0;
+    ChunkFetch f;
+    if ((uint32_t)w < ntot) fetch_chunk(bb, col, pol, NL, NLC, ES, (uint32_t)w, lane, below, lcur, f);
+    for (uint32_t c = (uint32_t)w; c < ntot; c += kWarps) {
+        int32_t u[4];
+        uint32_t nd[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            u[k] = ((f.vm >> k) & 1u) ? f.u[k] : -1;
+            nd[k] = f.nd[k];
+        }
+        uint32_t pv[4];
+        if constexpr (ATOS_CHUNK_PIPE == 1)
+            if (c + kWarps < ntot) fetch_chunk(bb, col, pol, NL, NLC, ES, c + kWarps, lane, below, lcur, f);
+        if constexpr (VIS) probe_vis<4>(s, kp, hcs, u, pv, hits);
+        else probe_bfs1<4>(s, kp, hcs, u, nd, pv, hits);
+        if constexpr (ATOS_CHUNK_PIPE != 1)
+            if (c + kWarps < ntot) fetch_chunk(bb, col, pol, NL, NLC, ES, c + kWarps, lane, below, lcur, f);
+        uint32_t msk;
+        if constexpr (VIS) finish_vis<4>(s, kp, u, s.pq_th, pv, msk);
+        else finish_bfs1<4>(s, u, nd, pv, msk);
+        if (__any_sync(kFull, msk != 0)) {
+            uint32_t item[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) item[k] = pq_tag((uint32_t)(u[k] - vb), nd[k], s.pq_th);
+            warp_append_mask<4>(s, w, wn, msk, item, kp.relax_red);
+        }
+    }
+    if (kp.hub_n) {
+        hits = __reduce_add_sync(kFull, hits);
+        if (lane == 0 && hits) atomicAdd(&s.c_hub, (unsigned long long)hits);
     }
 }
 
@@ -467,8 +590,13 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     if (NLC + ES > 0) {
         const int w = tid >> 5;
         uint32_t wn = s.wn[w];
-        if (kp.vis) expand_bfs1<true>(s, bb, kp, NL, NLC, ES, wn);
-        else expand_bfs1<false>(s, bb, kp, NL, NLC, ES, wn);
+        if constexpr (ATOS_CHUNK_PIPE != 0 && kLongG == 1) {
+            if (kp.vis) expand_bfs1_pipe<true>(s, bb, kp, NL, NLC, ES, wn);
+            else expand_bfs1_pipe<false>(s, bb, kp, NL, NLC, ES, wn);
+        } else {
+            if (kp.vis) expand_bfs1<true>(s, bb, kp, NL, NLC, ES, wn);
+            else expand_bfs1<false>(s, bb, kp, NL, NLC, ES, wn);
+        }
         __syncwarp();
         if ((tid & 31) == 0) s.wn[w] = wn;
     }

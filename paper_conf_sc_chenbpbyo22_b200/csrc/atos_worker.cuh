@@ -169,11 +169,16 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return m;
 }
 
+// Rank owning global vertex u: the largest r with part[r] <= u (binary search;
+// an unrolled scan over all kMaxRanks entries was 12 % of the 8-rank BFS
+// worker's instructions).
 __device__ __forceinline__ int owner_of(const RankDev &R, int64_t u) {
-    int r = 0;
-#pragma unroll
-    for (int k = 1; k < kMaxRanks; ++k) r += (k < R.n_ranks && R.part[k] <= u) ? 1 : 0;
-    return r;
+    int lo = 0, hi = R.n_ranks - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (R.part[mid] <= u) lo = mid; else hi = mid - 1;
+    }
+    return lo;
 }
 
 // Dynamic shared memory after Smem: the BFS hub bounds (atos_bfs1.cuh).
@@ -469,14 +474,18 @@ __device__ __noinline__ uint32_t warp_flush_remote(Smem &s, const KParams &kp, i
 template <int APP>
 __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, int cta, int w, bool pred, int dst,
                                                    uint32_t v_local, uint64_t payload, uint32_t &wn) {
-    const RankDev &R = s.R;
-    if (__ballot_sync(kFull, pred) == 0) return;
+    uint32_t todo = __ballot_sync(kFull, pred);
+    if (todo == 0) return;
     const int lane = threadIdx.x & 31;
     const uint32_t mask = (uint32_t)(kp.stage_cap - 1);
-    for (int d = 0; d < R.n_ranks; ++d) {
+    // one round per destination present among the lanes (a loop over all
+    // n_ranks destinations with a ballot each was 38 % of the 8-rank BFS
+    // worker's instructions)
+    while (todo) {
+        const int d = __shfl_sync(kFull, dst, __ffs(todo) - 1);
         const bool mine = pred && dst == d;
         const uint32_t m = __ballot_sync(kFull, mine);
-        if (m == 0) continue;
+        todo &= ~m;
         __syncwarp();
         if (s.wst[w][d] - s.wsh[w][d] + 32 > (uint32_t)kp.stage_cap) {
             // full packets out first (keeps room for this row)
