@@ -92,11 +92,13 @@ typedef struct {
                                  each 32-edge step produced at once (Listing
                                  5's per-warp push; packets of <= 32
                                  messages)                                    */
-    int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE)      */
+    int32_t agg_batch_msgs;   /* packet size in messages (the BATCH_SIZE);
+                                 default 1024 (channel sweep)      */
     int64_t agg_max_age_ns;   /* flush age (the WAIT_TIME) in ns of
                                  %globaltimer, checked at batch end and when
                                  idle                                          */
-    int32_t channel_packets;  /* packets per (src->dst) channel ring, pow2    */
+    int32_t channel_packets;  /* packets per (src->dst) channel ring, pow2;
+                                 default 4096                                  */
     int64_t watchdog_ms;      /* device watchdog per solve; 0 = none           */
     int32_t rank;             /* SPMD: this process's rank                     */
     int32_t n_ranks;          /* SPMD: number of processes (1 = single GPU)    */

@@ -89,9 +89,12 @@ extern "C" atos_status atos_config_init(atos_config *cfg) {
     cfg->probe_filter = 2;
     cfg->ring_cap_factor = 2.0;
     cfg->agg_enabled = 1;
-    cfg->agg_batch_msgs = 256;
+    // channel sweep, virtual ranks: PR RMAT-20 at 2 ranks 132 -> 59 ms with
+    // 4096 packets per channel (senders stalled on full channels at batch end), 50 ms with
+    // 1024-message packets; 8 ranks 115 -> 108 ms; BFS within noise
+    cfg->agg_batch_msgs = 1024;
     cfg->agg_max_age_ns = 4000;      // ~the paper's eager WAIT_TIME for BFS
-    cfg->channel_packets = 1024;
+    cfg->channel_packets = 4096;
     cfg->watchdog_ms = 60000;
     cfg->rank = 0;
     cfg->n_ranks = 1;
@@ -214,8 +217,11 @@ static Layout make_layout(const Shape &S, const int64_t *part, int r) {
 // sub-channels per channel: about 8 inbound cursors per rank in total (a single
 // cursor serialised the receive side at 2 ranks), each sub-channel >= 2 packets
 static int nsub_for(int p, int cp) {
+    // about `rings` inbound rings per rank in total (ATOS_INBOUND_RINGS: A/B switch,
+    // must be the same in every process of a multi-process run)
+    static const int rings = std::getenv("ATOS_INBOUND_RINGS") ? std::max(1, std::atoi(std::getenv("ATOS_INBOUND_RINGS"))) : 8;
     int k = 1;
-    while (k < kMaxSub && k * 2 * (p - 1) <= 8 && cp / (k * 2) >= 2) k *= 2;
+    while (k < kMaxSub && k * 2 * (p - 1) <= rings && cp / (k * 2) >= 2) k *= 2;
     return p > 1 ? k : 1;
 }
 

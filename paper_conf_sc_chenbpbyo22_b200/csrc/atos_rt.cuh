@@ -133,6 +133,12 @@ __device__ __forceinline__ uint64_t ld_acquire_peer(bool sys, const uint64_t *p)
 __device__ __forceinline__ uint64_t ld_relaxed_peer(bool sys, const uint64_t *p) {
     return sys ? ld_relaxed_sys(p) : ld_relaxed_gpu(p);
 }
+__device__ __forceinline__ uint32_t ld_relaxed_peer_u32(bool sys, const uint32_t *p) {
+    uint32_t v;
+    if (sys) asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    else asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
 __device__ __forceinline__ void st_release_peer(bool sys, uint64_t *p, uint64_t v) {
     if (sys) st_release_sys(p, v); else st_release_gpu(p, v);
 }

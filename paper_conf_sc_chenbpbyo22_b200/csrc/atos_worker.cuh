@@ -518,6 +518,64 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
 constexpr int kClaim = 8;
 constexpr int kInU = 4;              // messages per lane in flight while applying
 
+#ifndef ATOS_INBOUND_WIDE
+// experiment, off: 1 = poll every inbound channel at once (inbound_claim_wide).
+// Measured slower (virtual ranks, same box: PR RMAT-20 2/4/8 ranks 51/75/109 ->
+// 83/140/254 ms, BFS RMAT-24 2/8 ranks 10.9/20.6 -> 11.9/23.4 ms): every idle
+// worker then claims the first ready channel in the same rotation order, and the
+// claims collide on its cursor
+#define ATOS_INBOUND_WIDE 0
+#endif
+
+// Whole warp, up to 32 inbound sub-channels (nc <= 32): poll them all at once --
+// lane l takes channel (start + l) mod nc, loads its cursor, then the sequence
+// words of its next kClaim packet headers (independent loads) -- pick the first
+// channel (in rotation order) with a ready prefix and claim that prefix with ONE
+// CAS on its cursor.  Two load round trips to look at every channel, where the
+// one-by-one walk took two per channel (an idle 8-rank worker walked 7 channels,
+// ~14 round trips, while the other 15 warps waited at the inbound barrier).
+// Returns the claimed packet count (0: nothing claimed) with the channel and the
+// cursor value; the caller acquires the claimed headers.
+__device__ __forceinline__ int inbound_claim_wide(const Smem &s, const KParams &kp, int start, int &ch_out,
+                                                  uint64_t &cc_out) {
+    const RankDev &R = s.R;
+    const int lane = threadIdx.x & 31;
+    const int nc = R.n_ranks * kp.nsub;
+    int ch = start + lane;
+    if (ch >= nc) ch -= nc;
+    const int sr = ch / kp.nsub, sk = ch - sr * kp.nsub;
+    const bool valid = lane < nc && sr != R.rank;
+    int r = 0;
+    uint64_t cc = 0;
+    if (valid) {
+        cc = ld_relaxed_gpu(&R.ctrl->in_cursor[ch].v);
+        const int lim = kClaim < kp.cps ? kClaim : kp.cps;
+        uint32_t sq[kClaim];
+#pragma unroll
+        for (int k = 0; k < kClaim; ++k)     // the header's high word: the packet's sequence tag
+            sq[k] = k < lim ? ld_relaxed_peer_u32(kp.sys, reinterpret_cast<const uint32_t *>(
+                                                            &R.in_hdr[sr][sub_slot(kp, sk, cc + k)]) + 1)
+                            : 0u;
+#pragma unroll
+        for (int k = 0; k < kClaim; ++k)
+            if (r == k && k < lim && sq[k] == lo32(cc + k + 1)) r = k + 1;
+    }
+    const uint32_t m = __ballot_sync(kFull, r > 0);
+    if (m == 0) return 0;
+    const int src = __ffs(m) - 1;
+    const int rr = __shfl_sync(kFull, r, src);
+    const uint64_t c2 = __shfl_sync(kFull, cc, src);
+    const int chs = __shfl_sync(kFull, ch, src);
+    int won = 0;
+    if (lane == 0)
+        won = atomicCAS((unsigned long long *)&R.ctrl->in_cursor[chs].v, (unsigned long long)c2,
+                        (unsigned long long)(c2 + (uint64_t)rr)) == c2;
+    if (!__shfl_sync(kFull, won, 0)) return 0;
+    ch_out = chs;
+    cc_out = c2;
+    return rr;
+}
+
 template <int APP>
 __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
     const RankDev &R = s.R;
@@ -526,31 +584,43 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
     const uint32_t cps = (uint32_t)kp.cps;
     const int p = R.n_ranks, nc = p * kp.nsub;
     const int start = (w + (int)(s.c_idle & 7)) % nc;
-    for (int kk = 0; kk < nc; ++kk) {
-        const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
-        if (sr == R.rank) continue;
-        unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+    const bool wide = ATOS_INBOUND_WIDE && nc <= 32;
+    // (channel ch = sr * nsub + sk walked incrementally: a div / mod per probed
+    // channel was a third of a polling sender's instructions)
+    int sr0 = start / kp.nsub, sk0 = start - sr0 * kp.nsub;
+    for (int kk = 0; kk < (wide ? 1 : nc);
+         ++kk, (++sk0 == kp.nsub) ? (sk0 = 0, sr0 = (sr0 + 1 == p ? 0 : sr0 + 1)) : 0) {
+        int sr = sr0, sk = sk0, ch = sr * kp.nsub + sk, r = 0;
         uint64_t cc = 0;
-        if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
-        cc = __shfl_sync(kFull, cc, 0);
-        bool ready = false;
         uint32_t cnt = 0;
-        if (lane < kClaim && (uint32_t)lane < cps) {
-            // relaxed poll: an acquire load also invalidates L1 (CCTL.IVALL), which
-            // every idle warp would otherwise do on every poll of every channel
-            const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);
-            ready = hi32(h) == lo32(cc + lane + 1);
-            cnt = lo32(h);
+        if (wide) {
+            r = inbound_claim_wide(s, kp, start, ch, cc);
+            if (r == 0) return false;
+            sr = ch / kp.nsub;
+            sk = ch - sr * kp.nsub;
+        } else {
+            if (sr == R.rank) continue;
+            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+            if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+            cc = __shfl_sync(kFull, cc, 0);
+            bool ready = false;
+            if (lane < kClaim && (uint32_t)lane < cps) {
+                // relaxed poll: an acquire load also invalidates L1 (CCTL.IVALL), which
+                // every idle warp would otherwise do on every poll of every channel
+                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);
+                ready = hi32(h) == lo32(cc + lane + 1);
+            }
+            const uint32_t nready = __ballot_sync(kFull, ready);
+            r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;   // ready prefix
+            if (r == 0) continue;
+            int won = 0;
+            if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+            if (!__shfl_sync(kFull, won, 0)) continue;
         }
-        const uint32_t nready = __ballot_sync(kFull, ready);
-        const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;   // ready prefix
-        if (r == 0) continue;
-        int won = 0;
-        if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
-        if (!__shfl_sync(kFull, won, 0)) continue;
-        // acquire each claimed header (synchronises with its sender's st.release),
-        // then the warp barrier orders every lane's payload reads after them
-        if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);
+        // acquire each claimed header (synchronises with its sender's st.release;
+        // its low word is the packet's message count), then the warp barrier
+        // orders every lane's payload reads after them
+        if (lane < r) cnt = lo32(ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]));
         __syncwarp();
         uint32_t total = 0;
         for (int q = 0; q < r; ++q) {
@@ -637,27 +707,36 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
         const int nc = R.n_ranks * kp.nsub;
         const int start = (cta + (int)s.c_idle) % nc;
         int got = 0;
-        for (int kk = 0; kk < nc && !got; ++kk) {
-            const int ch = (start + kk) % nc, sr = ch / kp.nsub, sk = ch % kp.nsub;
-            if (sr == R.rank) continue;
-            unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+        const bool wide = ATOS_INBOUND_WIDE && nc <= 32;     // one look at every channel (inbound_claim_wide)
+        int sr0 = start / kp.nsub, sk0 = start - sr0 * kp.nsub;
+        for (int kk = 0; kk < (wide ? 1 : nc) && !got;
+             ++kk, (++sk0 == kp.nsub) ? (sk0 = 0, sr0 = (sr0 + 1 == R.n_ranks ? 0 : sr0 + 1)) : 0) {
+            int sr = sr0, sk = sk0, ch = sr * kp.nsub + sk, r = 0;
             uint64_t cc = 0;
-            if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
-            cc = __shfl_sync(kFull, cc, 0);
-            bool ready = false;
-            uint32_t cnt = 0;
-            if (lane < kClaim && (uint32_t)lane < cps) {
-                const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
-                ready = hi32(h) == lo32(cc + lane + 1);
-                cnt = lo32(h);
+            if (wide) {
+                r = inbound_claim_wide(s, kp, start, ch, cc);
+                if (r == 0) break;
+                sr = ch / kp.nsub;
+                sk = ch - sr * kp.nsub;
+            } else {
+                if (sr == R.rank) continue;
+                unsigned long long *cur = (unsigned long long *)&R.ctrl->in_cursor[ch].v;
+                if (lane == 0) cc = ld_relaxed_gpu((const uint64_t *)cur);
+                cc = __shfl_sync(kFull, cc, 0);
+                bool ready = false;
+                if (lane < kClaim && (uint32_t)lane < cps) {
+                    const uint64_t h = ld_relaxed_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // relaxed poll
+                    ready = hi32(h) == lo32(cc + lane + 1);
+                }
+                const uint32_t nready = __ballot_sync(kFull, ready);
+                r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
+                if (r == 0) continue;
+                int won = 0;
+                if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
+                if (!__shfl_sync(kFull, won, 0)) continue;
             }
-            const uint32_t nready = __ballot_sync(kFull, ready);
-            const int r = (~nready == 0u) ? 32 : __ffs(~nready) - 1;
-            if (r == 0) continue;
-            int won = 0;
-            if (lane == 0) won = atomicCAS(cur, (unsigned long long)cc, (unsigned long long)(cc + r)) == cc;
-            if (!__shfl_sync(kFull, won, 0)) continue;
-            if (lane < r) (void)ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)]);   // sync with each sender's release
+            // sync with each sender's release; the header's low word is the message count
+            const uint32_t cnt = lane < r ? lo32(ld_acquire_peer(kp.sys, &R.in_hdr[sr][sub_slot(kp, sk, cc + lane)])) : 0u;
             uint32_t incl = lane < r ? cnt : 0u;
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
