@@ -471,17 +471,43 @@ __global__ void permute_rows_kernel(const int64_t *rp_old, const int32_t *col_ol
 // Streamed variant for a host column array: old rows [l0, l1) restricted to the
 // staged column range [c0, c1) (rank-relative offsets), one warp per old row;
 // column ids are range-checked here (they are never checked elsewhere on this path).
+// One warp per old row clipped to the chunk; a row with more than kPermLong
+// edges in the chunk is deferred to permute_long_kernel (one CTA per row), so a
+// hub row does not leave one warp running long after the rest of the grid (the
+// last chunk of RMAT-24 took 11.8 ms against ~5 ms for the others).
+constexpr int64_t kPermLong = 8192;
 __global__ void permute_chunk_kernel(const int64_t *rp_old, const int32_t *stage, int64_t c0, int64_t c1,
                                      int64_t l0, int64_t l1, const int32_t *perm, int64_t v0,
-                                     const int64_t *rp_new, int32_t *col_new, int64_t n, unsigned long long *bad) {
+                                     const int64_t *rp_new, int32_t *col_new, int64_t n, unsigned long long *bad,
+                                     int64_t *long_rows, unsigned int *n_long) {
     const int lane = threadIdx.x & 31;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t l = l0 + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); l < l1; l += nw) {
         const int64_t b = rp_old[l], e = rp_old[l + 1];
         const int64_t lo = b > c0 ? b : c0, hi = e < c1 ? e : c1;
         if (lo >= hi) continue;
+        if (hi - lo > kPermLong) {
+            if (lane == 0) long_rows[atomicAdd(n_long, 1u)] = l;
+            continue;
+        }
         const int64_t o = rp_new[perm[v0 + l] - v0] + (lo - b);
         for (int64_t k = lane; k < hi - lo; k += 32) {
+            int32_t x = stage[lo - c0 + k];
+            if (x < 0 || (int64_t)x >= n) { atomicOr(bad, 2ull); x = 0; }
+            col_new[o + k] = perm[x];
+        }
+    }
+}
+
+__global__ void permute_long_kernel(const int64_t *rp_old, const int32_t *stage, int64_t c0, int64_t c1,
+                                    const int32_t *perm, int64_t v0, const int64_t *rp_new, int32_t *col_new, int64_t n,
+                                    unsigned long long *bad, const int64_t *long_rows, const unsigned int *n_long) {
+    for (unsigned int i = blockIdx.x; i < *n_long; i += gridDim.x) {
+        const int64_t l = long_rows[i];
+        const int64_t b = rp_old[l], e = rp_old[l + 1];
+        const int64_t lo = b > c0 ? b : c0, hi = e < c1 ? e : c1;
+        const int64_t o = rp_new[perm[v0 + l] - v0] + (lo - b);
+        for (int64_t k = threadIdx.x; k < hi - lo; k += blockDim.x) {
             int32_t x = stage[lo - c0 + k];
             if (x < 0 || (int64_t)x >= n) { atomicOr(bad, 2ull); x = 0; }
             col_new[o + k] = perm[x];
@@ -609,6 +635,8 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     CU(dmalloc(g, &v0, (size_t)n * 4)); fr.p.push_back(v0);
     CU(dmalloc(g, &d_max, 8)); fr.p.push_back(d_max);
     CU(cudaMemsetAsync(d_max, 0, 8, st));
+    LoadTrace tr;
+    tr.mark(st, "  relabel: row_ptr + scratch");
     degree_keys_kernel<<<1024, 256, 0, st>>>(rpf, n, k0, v0, d_max);
     CU(cudaGetLastError());
     unsigned long long mx = 0;
@@ -618,6 +646,7 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     g->skewed = (double)mx >= 32.0 * std::max(1.0, mean);
     if (g->cfg.relabel == 0) return ATOS_OK;                           // degree statistics only
     if (g->cfg.relabel == 2 && !g->skewed) return ATOS_OK;              // not skewed: keep the given order
+    tr.mark(st, "  relabel: degree keys");
     CU(dmalloc(g, &g->d_inv, (size_t)n * 4));
     CU(dmalloc(g, &g->d_perm, (size_t)n * 4));
     int64_t maxlen = 0;
@@ -633,6 +662,7 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
         size_t t2 = tb;
         CU(cub::DeviceRadixSort::SortPairs(tmp, t2, k0 + b, k1 + b, v0 + b, g->d_inv + b, (int)len, 0, 32, st));
     }
+    tr.mark(st, "  relabel: sort");
     invert_perm_kernel<<<1024, 256, 0, st>>>(g->d_inv, n, g->d_perm);
     CU(cudaGetLastError());
     CU(cudaStreamSynchronize(st));
@@ -696,6 +726,10 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
     const int64_t CH = std::min<int64_t>(std::max<int64_t>(m, 1), ch);
     int32_t *stage[2] = {nullptr, nullptr};
     for (int k = 0; k < 2; ++k) { CU(dmalloc(g, &stage[k], (size_t)CH * 4)); fr.p.push_back(stage[k]); }
+    int64_t *long_rows = nullptr;            // rows deferred to permute_long_kernel (> kPermLong edges in a chunk)
+    unsigned int *n_long = nullptr;
+    CU(dmalloc(g, &long_rows, (size_t)(CH / kPermLong + 2) * 8)); fr.p.push_back(long_rows);
+    CU(dmalloc(g, &n_long, sizeof(unsigned int))); fr.p.push_back(n_long);
     cudaStream_t cs = nullptr;
     CU(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
     cudaEvent_t ev_in[2], ev_out[2], ev_ready;
@@ -731,8 +765,12 @@ static atos_status relabel_rows_streamed(atos_graph *g, LocalRank &me, const int
         cudaEventRecord(ev_in[b], cs);
         cudaStreamWaitEvent(st, ev_in[b], 0);
         tmark(st);
+        cudaMemsetAsync(n_long, 0, sizeof(unsigned int), st);
         permute_chunk_kernel<<<2048, 256, 0, st>>>(me.row_ptr, stage[b], c0, c1, std::max<int64_t>(l0, 0),
-                                                  std::min(l1, nr), g->d_perm, v0, rp_new, col_new, g->n, d_bad);
+                                                  std::min(l1, nr), g->d_perm, v0, rp_new, col_new, g->n, d_bad,
+                                                  long_rows, n_long);
+        permute_long_kernel<<<1024, 512, 0, st>>>(me.row_ptr, stage[b], c0, c1, g->d_perm, v0, rp_new, col_new, g->n,
+                                                 d_bad, long_rows, n_long);
         tmark(st);
         cudaEventRecord(ev_out[b], st);
     }
@@ -1061,6 +1099,9 @@ static KParams make_params(atos_graph *g) {
         // claim at pop (RED discoveries, one atomicOr per pop): RMAT-26 9.81 -> 8.62 ms,
         // RMAT-24 2.72 -> 2.43 ms; ATOS_VIS_NOCLAIM restores the discoverer's atomicOr (A/B)
         if (kp.vis && !std::getenv("ATOS_VIS_NOCLAIM")) kp.vis_claim = 1;
+        // next-batch reservation during the expansion (the leader's pop took ~5
+        // dependent round trips with the whole CTA waiting); ATOS_NO_PQ_EARLY (A/B)
+        kp.pq_early = kp.vis && !g->cfg.discrete && !std::getenv("ATOS_NO_PQ_EARLY");
     }
     kp.agg_age_ns = g->cfg.agg_max_age_ns;
     kp.watchdog_ns = g->cfg.watchdog_ms * 1000000ll;

@@ -587,6 +587,22 @@ __device__ void process_batch_bfs1(Smem &s, const KParams &kp, int cta, int B) {
     }
     if (hub && !(kp.hub_dbg & 2)) hub_copy_wait(s, s.hub_par ^ 1u);             // this batch's bounds have landed
     __syncthreads();
+    if (tid == 0 && kp.pq_early) {
+        // level buckets: reserve the NEXT batch on the current ring now, so the
+        // head atomic leaves the critical path between batches -- only when the
+        // ring holds plenty of work (a reservation withholds items from idle
+        // workers).  An early reservation is an ordinary one taken sooner: if the
+        // bucket advances first, pq_choose serves it as a stale one (pq_recycle).
+        const int q = s.pq_q;
+        uint64_t &lo = res_lo_q(s, q), &hi = res_hi_q(s, q);
+        if (lo == hi) {
+            const uint64_t t = ld_relaxed_gpu(q_tail(R, q)), h = ld_relaxed_gpu(q_head(R, q));
+            if (t > h && t - h >= 2ull * (uint64_t)kp.ctas_per_rank * (uint64_t)kp.fetch) {
+                lo = atomicAdd((unsigned long long *)q_head(R, q), (unsigned long long)kp.fetch);
+                hi = lo + (uint64_t)kp.fetch;
+            }
+        }
+    }
     if (NLC + ES > 0) {
         const int w = tid >> 5;
         uint32_t wn = s.wn[w];

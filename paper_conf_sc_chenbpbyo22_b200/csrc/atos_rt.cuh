@@ -326,6 +326,7 @@ struct KParams {
     int32_t discrete;        // discrete-kernel mode: pop only below ctrl->limit, exit when drained
     int32_t sys;             // peers are other devices/processes: system-scope ordering (else .gpu)
     int32_t early;           // reserve the next batch during expansion
+    int32_t pq_early;        // level buckets: reserve the next batch on the current ring during expansion
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming

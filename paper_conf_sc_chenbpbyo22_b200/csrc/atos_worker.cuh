@@ -138,6 +138,7 @@ struct alignas(16) Smem {
     uint64_t res2_lo, res2_hi;     // priority queue: outstanding reservation on ring 1
     uint64_t ring2_base;           // ring 1 tail at the start of this solve
     uint64_t pq_st;                // priority queue: pq_state read at the last pop
+    uint64_t pq_k0;                // priority queue: pq_state at the start of the solve (Ctrl::pq_k0)
     uint32_t pq_th;                // current threshold (kNoTh: FIFO, nothing is far)
     int32_t pq_q;                  // current ring (pq_state & 1; 0 without the priority queue)
     int32_t pop_q;                 // ring the current batch was popped from
@@ -1517,7 +1518,7 @@ __device__ __noinline__ void pq_choose(Smem &s, const KParams &kp) {
     const RankDev &R = s.R;
     const uint64_t st = ld_relaxed_gpu(&R.ctrl->pq_state.v);
     const int q = (int)(st & 1);
-    const uint64_t k = st - ld_relaxed_gpu(&R.ctrl->pq_k0.v);
+    const uint64_t k = st - s.pq_k0;
     const uint64_t th = (uint64_t)kp.pq_th0 + k * (uint64_t)kp.pq_delta;
     s.pq_st = st;
     s.pq_q = q;
@@ -1728,9 +1729,11 @@ __device__ __forceinline__ void worker_body(Smem &s, const KParams &kp) {
         s.pq_q = s.pop_q = 0;
         s.pq_st = 0;
         s.pq_th = kNoTh;
+        s.pq_k0 = 0;
         if (kp.pq) {        // the bucket at the start of the launch (pop_batch re-reads it)
             const uint64_t st = ld_relaxed_gpu(&s.R.ctrl->pq_state.v);
-            const uint64_t th = (uint64_t)kp.pq_th0 + (st - ld_relaxed_gpu(&s.R.ctrl->pq_k0.v)) * (uint64_t)kp.pq_delta;
+            s.pq_k0 = ld_relaxed_gpu(&s.R.ctrl->pq_k0.v);      // fixed for the solve (seed kernel)
+            const uint64_t th = (uint64_t)kp.pq_th0 + (st - s.pq_k0) * (uint64_t)kp.pq_delta;
             s.pq_q = s.pop_q = (int)(st & 1);
             s.pq_th = th < (uint64_t)kNoTh ? (uint32_t)th : kNoTh - 1;
         }

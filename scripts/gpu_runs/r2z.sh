@@ -12,3 +12,5 @@ bash scripts/gpu_prof.sh ${T}_bfs24 bfs rmat24
 bash scripts/gpu_prof.sh ${T}_bfs26 bfs rmat26
 bash scripts/gpu_prof.sh ${T}_pr20 pr
 tail -3 gpurun_out/$T/pytest.log gpurun_out/$T/smoke.log; head -c 400 gpurun_out/$T/bench.json
+bash scripts/gpu_prof.sh ${T}_pr20vr8 pr rmat20_pr '{"virtual_ranks":8, "relabel":0}'
+bash scripts/gpu_prof.sh ${T}_bfs24vr8 bfs rmat24 '{"virtual_ranks":8}'

@@ -320,6 +320,24 @@ def test_streamed_relabel_load_from_host(chunk, monkeypatch):
     assert e.value.status == 1
 
 
+@pytest.mark.parametrize("chunk", ["100003", "30000"])
+def test_streamed_relabel_long_rows(chunk, monkeypatch):
+    """Rows with more than 8192 edges inside one load chunk go to the one-CTA-per-row
+    permutation kernel (graph_load's streamed relabeling)."""
+    monkeypatch.setenv("ATOS_LOAD_CHUNK", chunk)
+    n = 40000
+    hub = torch.zeros(n - 1, dtype=torch.int64)
+    leaves = torch.arange(1, n, dtype=torch.int64)
+    chain = torch.arange(1, n - 1, dtype=torch.int64)
+    src_e = torch.cat([hub, chain, torch.full((n - 2,), 7, dtype=torch.int64)])
+    dst_e = torch.cat([leaves, chain + 1, torch.arange(2, n, dtype=torch.int64)])
+    keep = src_e != dst_e
+    rp, col = inputs.csr_from_edges(n, src_e[keep], dst_e[keep], symmetrize=True).numpy()
+    assert np.diff(rp).max() > 3 * 8192
+    for s in (0, 123, n - 1):
+        run_and_check(rp, col, s, relabel=1)
+
+
 def bfs_properties_hold(rp_dev, col_dev, depth_dev, src):
     """Properties that fix BFS depths on a symmetric graph at any size (checked on
     the GPU with plain torch ops): depth(src) = 0; |d(u) - d(v)| <= 1 on every edge

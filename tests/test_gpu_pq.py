@@ -131,7 +131,7 @@ def test_pq_rmat24_config2_full_size():
     assert st["edges"] == m_reached(rp, d)
 
 
-@pytest.mark.parametrize("var", ["ATOS_VIS_NOCLAIM", "ATOS_NO_VIS"])
+@pytest.mark.parametrize("var", ["ATOS_VIS_NOCLAIM", "ATOS_NO_VIS", "ATOS_NO_PQ_EARLY"])
 def test_pq_delta1_switches(monkeypatch, var):
     # the level-bucket variants behind the A/B switches: discoverer
     # atomicOr instead of claim at pop; depth words + filter instead of the bitmap
