@@ -711,11 +711,19 @@ def other_configs(args, dev, stream, cfg, load, world):
                                                                        os.environ.get("ATOS_SAME_DEVICE") else "")
         c5 = {"workload": f"configs[4] PageRank alpha=.85 eps=1e-9, RMAT-26 ef16 directed, {ranks}",
               "n": g.n, "nnz": g.nnz}
+        # delta messages with aggregation on / off / N2 combining (the paper's comparison), and on
+        # virtual ranks also the default there: remote atomics + activation messages for crossings
         modes = (("agg_on", 1, 0, 0), ("agg_off", 0, 0, 0), ("agg_on_combine_N2", 1, 1, 0))
-        for name, agg, comb, _ in modes:
+        if world == 1:
+            modes += (("remote_atomics_activations", 1, 0, 1),)
+        for name, agg, comb, ratom in modes:
             extra = dict(relabel=0, agg_enabled=agg, pr_combine=comb)
             if world == 1:
                 extra["virtual_ranks"] = 8
+            if ratom:
+                os.environ.pop("ATOS_PR_NORATOM", None)
+            else:
+                os.environ["ATOS_PR_NORATOM"] = "1"     # (read per solve by libatos)
             P = load(g.row_ptr, g.col, g.n, **dict(cfg, **extra))
             if world > 1:
                 torch.distributed.barrier()
@@ -740,6 +748,7 @@ def other_configs(args, dev, stream, cfg, load, world):
             if world > 1:
                 torch.distributed.barrier()
             P.free()
+        os.environ.pop("ATOS_PR_NORATOM", None)
         out["rmat26_pr_8ranks" if world in (1, 8) else f"rmat26_pr_{world}ranks"] = c5
         del g, r_out, s_out
     return out

@@ -261,6 +261,8 @@ struct atos_graph {
     int32_t *d_depth_full = nullptr;
     int32_t *d_perm = nullptr;     // degree relabeling: old -> new (NULL = identity)
     int32_t *d_inv = nullptr;      //                    new -> old
+    int64_t *rp_dev_tmp = nullptr; // graph_load from host: device copy of the whole row_ptr made by
+                                   // compute_relabel, reused for the ranks' rows, freed at the end of load
     int hub_n = 0;                 // BFS hub bounds: ids [0, hub_n) covered (single rank, relabeled graphs)
     int hub_chunks = 0;            // hub_n / 128 rounded up to a multiple of 16 (array size)
     bool skewed = true;            // max degree >= 32 x mean degree (set when an auto option needs it)
@@ -311,14 +313,71 @@ static cudaMemPool_t pool_of(int device) {
     }
     return pools[device];
 }
+// Exact-size cache of large blocks for handles with pool_retain = 1 (load/solve/free
+// loops).  The pool alone kept the memory mapped but re-split it differently from one
+// load to the next, and a request that no longer fit mapped new memory synchronously
+// inside cudaMallocFromPoolAsync (40-800 ms stalls in random load phases, e2e trace).
+// A retained handle's large blocks are parked here at free and handed out again for
+// the same size; a handle with pool_retain = 0 empties the cache at its free.
+constexpr size_t kCacheMin = (size_t)64 << 20;
+struct BlockCache {
+    std::mutex mu;
+    std::vector<std::pair<size_t, void *>> parked;     // free blocks
+    std::vector<std::pair<void *, size_t>> sizes;      // every cacheable block handed out
+};
+static BlockCache &block_cache(int device) {
+    static BlockCache c[64];
+    return c[device & 63];
+}
 template <typename T>
 static cudaError_t dmalloc(const atos_graph *g, T **p, size_t bytes) {
+    const bool cache = g->cfg.pool_retain && bytes >= kCacheMin;
+    if (cache) {
+        BlockCache &c = block_cache(g->cfg.device);
+        std::lock_guard<std::mutex> lk(c.mu);
+        for (size_t i = 0; i < c.parked.size(); ++i)
+            if (c.parked[i].first == bytes) {
+                *p = (T *)c.parked[i].second;
+                c.parked.erase(c.parked.begin() + (long)i);
+                return cudaSuccess;
+            }
+    }
     cudaMemPool_t pool = pool_of(g->cfg.device);
-    if (!pool) return cudaMallocAsync((void **)p, bytes, g->stream);
-    return cudaMallocFromPoolAsync((void **)p, bytes, pool, g->stream);
+    const cudaError_t e = pool ? cudaMallocFromPoolAsync((void **)p, bytes, pool, g->stream)
+                               : cudaMallocAsync((void **)p, bytes, g->stream);
+    if (e == cudaSuccess && cache) {
+        BlockCache &c = block_cache(g->cfg.device);
+        std::lock_guard<std::mutex> lk(c.mu);
+        c.sizes.emplace_back((void *)*p, bytes);
+    }
+    return e;
 }
 static void dfree(const atos_graph *g, void *p) {
-    if (p) cudaFreeAsync(p, g->stream);
+    if (!p) return;
+    if (g->cfg.pool_retain) {
+        BlockCache &c = block_cache(g->cfg.device);
+        std::lock_guard<std::mutex> lk(c.mu);
+        for (const auto &x : c.sizes)
+            if (x.first == p) {
+                // the next user may be another handle on another stream: the block is
+                // parked only once this handle's pending work on it is done
+                cudaStreamSynchronize(g->stream);
+                c.parked.emplace_back(x.second, p);
+                return;
+            }
+    }
+    cudaFreeAsync(p, g->stream);
+}
+// Release every parked block (a handle without pool_retain is being freed).
+static void block_cache_release(const atos_graph *g) {
+    BlockCache &c = block_cache(g->cfg.device);
+    std::lock_guard<std::mutex> lk(c.mu);
+    for (const auto &x : c.parked) {
+        cudaFreeAsync(x.second, 0);     // (the handle's own stream may already be destroyed)
+        for (size_t i = 0; i < c.sizes.size(); ++i)
+            if (c.sizes[i].first == x.second) { c.sizes.erase(c.sizes.begin() + (long)i); break; }
+    }
+    c.parked.clear();
 }
 
 // dynamic shared memory of the worker: Smem, plus the BFS hub cache (one nibble per entry)
@@ -567,6 +626,7 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     dfree(g, g->d_depth_full);
     dfree(g, g->d_perm);
     dfree(g, g->d_inv);
+    dfree(g, g->rp_dev_tmp);
     dfree(g, g->d_accs);
     if (g->stream) cudaStreamSynchronize(g->stream);
     for (int a = 0; a < 2; ++a) {
@@ -579,8 +639,11 @@ extern "C" atos_status atos_graph_free(atos_graph *g) {
     if (g->ev_w1) cudaEventDestroy(g->ev_w1);
     if (g->ev_end) cudaEventDestroy(g->ev_end);
     if (g->own_stream && g->stream) cudaStreamDestroy(g->stream);
-    if (!g->cfg.pool_retain)
+    if (!g->cfg.pool_retain) {
+        block_cache_release(g);
+        cudaDeviceSynchronize();
         if (cudaMemPool_t pool = pool_of(g->cfg.device)) cudaMemPoolTrimTo(pool, 0);   // freed memory back to the device
+    }
     delete g;
     return ATOS_OK;
 }
@@ -623,7 +686,7 @@ static atos_status compute_relabel(atos_graph *g, const int64_t *row_ptr, bool r
     if (!rp_dev) {
         int64_t *t = nullptr;
         CU(dmalloc(g, &t, (size_t)(n + 1) * 8));
-        fr.p.push_back(t);
+        g->rp_dev_tmp = t;     // (graph_load copies the ranks' rows from it and frees it)
         CU(cudaMemcpyAsync(t, row_ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, st));
         rpf = t;
     }
@@ -923,7 +986,8 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         const bool streamed = g->d_perm && me.m_r > 0 && !rp_dev && !is_device_ptr(col) && !(se && se[0] == '0');
         CU(dmalloc(g, &me.row_ptr, (size_t)(nr + 1) * 8));
         if (!streamed) CU(dmalloc(g, &me.col, ((size_t)me.m_r + kColPad) * 4));
-        CU(cudaMemcpyAsync(me.row_ptr, row_ptr + g->part[r], (size_t)(nr + 1) * 8, cudaMemcpyDefault, g->stream));
+        CU(cudaMemcpyAsync(me.row_ptr, (g->rp_dev_tmp ? g->rp_dev_tmp : row_ptr) + g->part[r], (size_t)(nr + 1) * 8,
+                           cudaMemcpyDefault, g->stream));
         if (me.m_r > 0 && !streamed)
             CU(cudaMemcpyAsync(me.col, col + rb[r], (size_t)me.m_r * 4, cudaMemcpyDefault, g->stream));
         tr.mark(g->stream, "copy csr");
@@ -969,6 +1033,8 @@ extern "C" atos_status atos_graph_load(const int64_t *row_ptr, const int32_t *co
         }
         CU(cudaGetLastError());
     }
+    dfree(g, g->rp_dev_tmp);
+    g->rp_dev_tmp = nullptr;
     unsigned long long bad = 0;
     CU(cudaMemcpyAsync(&bad, d_bad, sizeof(bad), cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
@@ -1069,6 +1135,14 @@ static KParams make_params(atos_graph *g) {
     if (const char *e = std::getenv("ATOS_TIMELINE")) kp.timeline_ns = std::atoll(e) * 1000;   // experiment
     kp.split = g->cfg.split_edges < 0 ? kSplitAuto : g->cfg.split_edges;
     kp.combine = g->p > 1 && g->S.combine;
+    // multi-rank PR with remote atomics: a delta for a remote vertex is added in the owner's
+    // memory by the sender (one-sided atomic with return) and only a crossing of eps becomes a
+    // message (PR RMAT-20, 2/4/8 virtual ranks: 56/84/121 -> 41/47/61 ms, same box; messages
+    // 725 M -> 16 M at 2 ranks).  Virtual ranks only: their state is initialised before the one
+    // grid starts, while separate processes would need a barrier between every rank's init and
+    // any rank's first remote add, and cross-GPU atomics at system scope on every residual
+    // update (the owner's own adds included).  ATOS_PR_NORATOM sends delta messages (A/B).
+    kp.pr_ratom = g->p > 1 && !g->multiproc && !kp.combine && !std::getenv("ATOS_PR_NORATOM") ? 1 : 0;
     kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
     // early next-batch reservation + per-warp enqueue: measured within noise
     // (RMAT-24/26 BFS, RMAT-20 PR); off unless ATOS_EARLY is set (experiment)

@@ -182,6 +182,11 @@ __device__ __forceinline__ double atom_add_f64(double *p, double x) {
     asm volatile("atom.global.add.f64 %0, [%1], %2;" : "=d"(o) : "l"(p), "d"(x));
     return o;
 }
+__device__ __forceinline__ double atom_add_f64_sys(double *p, double x) {
+    double o;
+    asm volatile("atom.sys.global.add.f64 %0, [%1], %2;" : "=d"(o) : "l"(p), "d"(x));
+    return o;
+}
 __device__ __forceinline__ void red_add_f64(double *p, double x) {
     asm volatile("red.global.add.f64 [%0], %1;" ::"l"(p), "d"(x));
 }
@@ -327,6 +332,7 @@ struct KParams {
     int32_t sys;             // peers are other devices/processes: system-scope ordering (else .gpu)
     int32_t early;           // reserve the next batch during expansion
     int32_t pq_early;        // level buckets: reserve the next batch on the current ring during expansion
+    int32_t pr_ratom;        // multi-rank PR: remote deltas applied by atomics in the owner's memory, messages only for crossings
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming
@@ -377,6 +383,9 @@ __device__ __forceinline__ bool pq_is_far(uint32_t item) { return (item & (0x800
 // hubs, which receive most of the fp64 atomicAdds -- fall into different 32-B
 // sectors and L2 slices instead of serialising in one atomic unit.  A bijection.
 __host__ __device__ __forceinline__ int64_t pr_q_of(int64_t n_r) { return n_r >= 64 ? n_r / 8 : 0; }
+// PR message payload meaning "the delta was already added in the owner's memory and crossed eps:
+// enqueue the vertex" (KParams::pr_ratom); a real delta is never this NaN pattern
+constexpr uint64_t kPrActivate = ~0ull;
 __device__ __forceinline__ int64_t pr_slot(int64_t i, int64_t q) {
     return (q > 0 && i < 8 * q) ? (i & 7) * q + (i >> 3) : i;
 }

@@ -663,9 +663,14 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                         ul[j] = m[j].x;
                         pred[j] = false;
                         if (i < cq) {
-                            const double dlt = __longlong_as_double((long long)(((uint64_t)m[j].w << 32) | m[j].z));
-                            const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
-                            pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                            const uint64_t pv = ((uint64_t)m[j].w << 32) | m[j].z;
+                            if (pv == kPrActivate) {
+                                pred[j] = true;          // applied remotely by the sender (pr_ratom)
+                            } else {
+                                const double dlt = __longlong_as_double((long long)pv);
+                                const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
+                                pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                            }
                         }
                     }
                 }
@@ -780,9 +785,14 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                 } else {
                     const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
                     ul[j] = msg.x;
-                    const double dlt = __longlong_as_double((long long)(((uint64_t)msg.w << 32) | msg.z));
-                    const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
-                    pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                    const uint64_t pv = ((uint64_t)msg.w << 32) | msg.z;
+                    if (pv == kPrActivate) {
+                        pred[j] = true;                  // applied remotely by the sender (pr_ratom)
+                    } else {
+                        const double dlt = __longlong_as_double((long long)pv);
+                        const double old = atom_add_f64(R.pr_res + pr_slot(ul[j], R.pr_q), dlt);
+                        pred[j] = old < kp.eps && old + dlt >= kp.eps;
+                    }
                 }
             }
         }
@@ -1007,6 +1017,13 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                 } else if (comb && u[k] >= 0) {                      // combine into the ghost residual (N2)
                     const double old = atom_add_f64(R.pr_ghost + pr_slot(u[k], qn), dlt);
                     gcross[k] = old < kp.eps_g && old + dlt >= kp.eps_g;
+                } else if (MULTI && kp.pr_ratom && u[k] >= 0) {
+                    // remote delta applied in the owner's memory (one-sided atomic, the
+                    // paper's remote update); only a crossing becomes a message
+                    const int d = owner_of(R, u[k]);
+                    double *pr = R.peer_res[d] + pr_slot(u[k] - R.part[d], pr_q_of(R.part[d + 1] - R.part[d]));
+                    const double old = kp.sys ? atom_add_f64_sys(pr, dlt) : atom_add_f64(pr, dlt);
+                    gcross[k] = old < eps && old + dlt >= eps;
                 }
             }
             if constexpr (!multi) {
@@ -1028,6 +1045,12 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                         const int d = gcross[k] ? owner_of(R, u[k]) : 0;
                         warp_append_remote<APP>(s, kp, cta, w, gcross[k], d,
                                                 gcross[k] ? (uint32_t)(u[k] - R.part[d]) : 0u, gv, wn);
+                        continue;
+                    }
+                    if (kp.pr_ratom) {   // remote deltas already applied: activation messages for crossings only
+                        const int d = gcross[k] ? owner_of(R, u[k]) : 0;
+                        warp_append_remote<APP>(s, kp, cta, w, gcross[k], d,
+                                                gcross[k] ? (uint32_t)(u[k] - R.part[d]) : 0u, kPrActivate, wn);
                         continue;
                     }
                     const bool rem = u[k] >= 0 && !(u[k] >= vb && u[k] < ve);

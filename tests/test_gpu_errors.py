@@ -79,3 +79,25 @@ def test_free_returns_memory_to_the_device():
     torch.cuda.synchronize()
     free2, _ = torch.cuda.mem_get_info()
     assert free0 - free2 < 64 << 20, (free0, free1, free2)
+
+
+def test_retained_blocks_reused_then_released():
+    """pool_retain = 1 parks a freed handle's large blocks for the next load of the same
+    sizes (load/solve/free loops); results stay exact, and the next handle without
+    pool_retain returns everything to the device at its free."""
+    g = inputs.rmat(20, 16, 2, symmetric=True, device="cuda")
+    rp, col = g.numpy()
+    src = inputs.bfs_sources(g, 1)[0]
+    want = oracle.bfs(rp, col, src)
+    torch.cuda.synchronize()
+    free0, _ = torch.cuda.mem_get_info()
+    for _ in range(3):
+        G = atos.Graph(rp, col, pool_retain=1)          # host CSR: streamed load, several >= 64 MB blocks
+        assert np.array_equal(G.bfs(src), want)
+        G.free()
+    G = atos.Graph(g.row_ptr, g.col, g.n)
+    assert np.array_equal(G.bfs(src), want)
+    G.free()
+    torch.cuda.synchronize()
+    free1, _ = torch.cuda.mem_get_info()
+    assert free0 - free1 < 64 << 20, (free0, free1)

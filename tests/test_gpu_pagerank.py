@@ -82,12 +82,22 @@ def test_rmat14_directed():
     assert st["pops"] >= g.n
 
 
+@pytest.mark.parametrize("ratom", [True, False])
 @pytest.mark.parametrize("vr", [2, 4, 8])
 @pytest.mark.parametrize("agg", [0, 1])
-def test_virtual_ranks(vr, agg):
+def test_virtual_ranks(vr, agg, ratom, monkeypatch):
+    # ratom: remote deltas added in the owner's memory, activation messages for crossings
+    # (the virtual-rank default); else one delta message per remote relaxation
+    if not ratom:
+        monkeypatch.setenv("ATOS_PR_NORATOM", "1")
     g = inputs.rmat(13, 16, 1, symmetric=False)
     rp, col = g.numpy()
-    run_and_check(rp, col, virtual_ranks=vr, agg_enabled=agg, channel_packets=64)
+    _, st = run_and_check(rp, col, virtual_ranks=vr, agg_enabled=agg, channel_packets=64)
+    relax = st["edges"]
+    if ratom:
+        assert st["msgs_sent"] < 0.2 * relax, (st["msgs_sent"], relax)     # crossings only
+    else:
+        assert st["msgs_sent"] > 0.5 * relax * (vr - 1) / vr, (st["msgs_sent"], relax)
 
 
 def test_repeated_solves_one_handle():
@@ -128,10 +138,12 @@ def test_relabel_same_pagerank(opts):
 
 @pytest.mark.parametrize("vr", [2, 3, 8])
 @pytest.mark.parametrize("agg", [0, 1])
-def test_sender_side_combining(vr, agg):
+def test_sender_side_combining(vr, agg, monkeypatch):
     """ghost residual combining reaches the oracle's PageRank with
     fewer messages than sending every delta (deltas below eps / p are combined;
-    measured -40 % on RMAT-20 at 8 ranks)."""
+    measured -40 % on RMAT-20 at 8 ranks).  Compared with the delta-message
+    protocol (ATOS_PR_NORATOM), not with remote atomics + activations."""
+    monkeypatch.setenv("ATOS_PR_NORATOM", "1")
     g = inputs.rmat(13, 16, 1, symmetric=False)
     rp, col = g.numpy()
     _, st_plain = run_and_check(rp, col, virtual_ranks=vr, agg_enabled=agg, channel_packets=64)
