@@ -1143,6 +1143,11 @@ static KParams make_params(atos_graph *g) {
     // any rank's first remote add, and cross-GPU atomics at system scope on every residual
     // update (the owner's own adds included).  ATOS_PR_NORATOM sends delta messages (A/B).
     kp.pr_ratom = g->p > 1 && !g->multiproc && !kp.combine && !std::getenv("ATOS_PR_NORATOM") ? 1 : 0;
+    // multi-rank BFS the same way: a remote edge that improves the sender's ghost word lowers the
+    // owner's depth word with atomicMin and sends an activation only on an improvement there
+    // (RMAT-24 at 2/4/8 virtual ranks 12.2/16.5/21.6 -> 12.4/15.3/18.5 ms, same box; the grid at
+    // 4 ranks unchanged).  Virtual ranks only, as pr_ratom; ATOS_BFS_NORATOM (A/B)
+    kp.bfs_ratom = g->p > 1 && !g->multiproc && !std::getenv("ATOS_BFS_NORATOM") ? 1 : 0;
     kp.sys = g->multiproc ? 1 : 0;   // virtual ranks share this device: .gpu scope suffices
     // early next-batch reservation + per-warp enqueue: measured within noise
     // (RMAT-24/26 BFS, RMAT-20 PR); off unless ATOS_EARLY is set (experiment)

@@ -333,6 +333,7 @@ struct KParams {
     int32_t early;           // reserve the next batch during expansion
     int32_t pq_early;        // level buckets: reserve the next batch on the current ring during expansion
     int32_t pr_ratom;        // multi-rank PR: remote deltas applied by atomics in the owner's memory, messages only for crossings
+    int32_t bfs_ratom;       // multi-rank BFS: improvements applied by atomicMin in the owner's memory, activations only
     int32_t warp_flush;      // per-warp enqueue right after expansion (no keeping)
     int32_t edge_map;        // build the per-batch edge -> row bitmap map (batches <= kBitE edges)
     int32_t static_chunks;   // expand_warp: round-robin chunks per warp instead of claiming
@@ -386,6 +387,9 @@ __host__ __device__ __forceinline__ int64_t pr_q_of(int64_t n_r) { return n_r >=
 // PR message payload meaning "the delta was already added in the owner's memory and crossed eps:
 // enqueue the vertex" (KParams::pr_ratom); a real delta is never this NaN pattern
 constexpr uint64_t kPrActivate = ~0ull;
+// BFS message depth word flag: "the owner's depth word was already lowered to this depth by the
+// sender (KParams::bfs_ratom): enqueue the vertex"
+constexpr uint32_t kBfsActivate = 0x80000000u;
 __device__ __forceinline__ int64_t pr_slot(int64_t i, int64_t q) {
     return (q > 0 && i < 8 * q) ? (i & 7) * q + (i >> 3) : i;
 }

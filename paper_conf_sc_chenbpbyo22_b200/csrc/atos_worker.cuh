@@ -519,6 +519,26 @@ __device__ __forceinline__ void warp_append_remote(Smem &s, const KParams &kp, i
 constexpr int kClaim = 8;
 constexpr int kInU = 4;              // messages per lane in flight while applying
 
+// Multi-rank BFS, a remote edge that improved this rank's ghost word of u: send u's new depth
+// to its owner -- or, with bfs_ratom (virtual ranks), lower the owner's depth word here with one
+// atomicMin (the paper's remote update) and send an activation only if it improved
+// there.  Whole warp (warp_append_remote).
+template <int APP>
+__device__ __forceinline__ void bfs_send_remote(Smem &s, const KParams &kp, int cta, int w, bool rem, int64_t u,
+                                                uint32_t nd, uint32_t &wn) {
+    const RankDev &R = s.R;
+    const int d = rem ? owner_of(R, u) : 0;
+    uint64_t pay = nd;
+    if (kp.bfs_ratom) {
+        if (rem) {
+            const uint32_t ndw = dw_make(nd);
+            rem = atom_min_u32(R.peer_depth[d] + u, ndw) > ndw;
+        }
+        pay = nd | kBfsActivate;
+    }
+    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u - R.part[d]) : 0u, pay, wn);
+}
+
 #ifndef ATOS_INBOUND_WIDE
 // experiment, off: 1 = poll every inbound channel at once (inbound_claim_wide).
 // Measured slower (virtual ranks, same box: PR RMAT-20 2/4/8 ranks 51/75/109 ->
@@ -644,10 +664,15 @@ __device__ bool warp_inbound(Smem &s, const KParams &kp, int w, uint32_t &wn) {
                         ul[j] = lo32(m[j]);
                         pred[j] = false;
                         if (i < cq) {
-                            const uint32_t ndw = dw_make(hi32(m[j]));
-                            pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
-                            if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(m[j]));
-                            ul[j] = pq_tag(ul[j], hi32(m[j]), s.pq_th);
+                            const uint32_t hv = hi32(m[j]), dd = hv & ~kBfsActivate;
+                            if (hv & kBfsActivate) {
+                                pred[j] = true;          // lowered by the sender (bfs_ratom)
+                            } else {
+                                const uint32_t ndw = dw_make(dd);
+                                pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
+                            }
+                            if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], dd);
+                            ul[j] = pq_tag(ul[j], dd, s.pq_th);
                         }
                     }
                 } else {
@@ -778,10 +803,15 @@ __device__ bool cta_inbound(Smem &s, const KParams &kp, int cta) {
                 if constexpr (APP == kApBfs) {
                     const uint64_t msg = ld_cg_u64((const uint64_t *)pay + i);
                     ul[j] = lo32(msg);
-                    const uint32_t ndw = dw_make(hi32(msg));
-                    pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
-                    if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], hi32(msg));
-                    ul[j] = pq_tag(ul[j], hi32(msg), s.pq_th);
+                    const uint32_t hv = hi32(msg), dd = hv & ~kBfsActivate;
+                    if (hv & kBfsActivate) {
+                        pred[j] = true;                  // lowered by the sender (bfs_ratom)
+                    } else {
+                        const uint32_t ndw = dw_make(dd);
+                        pred[j] = atom_min_u32(R.depth + R.v_begin + ul[j], ndw) > ndw;
+                    }
+                    if (pred[j] && kp.filter) filt_put_fresh(R.filt, R.v_begin + ul[j], dd);
+                    ul[j] = pq_tag(ul[j], dd, s.pq_th);
                 } else {
                     const uint4 msg = ld_cg_u4((const uint4 *)pay + i);
                     ul[j] = msg.x;
@@ -986,10 +1016,7 @@ __device__ void expand_warp(Smem &s, BatchBuf &bb, const KParams &kp, int cta, i
                     const bool loc = imp[k] && u[k] >= vb && u[k] < ve;
                     if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
                     warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(u[k] - vb), nd[k], th));
-                    const bool rem = imp[k] && !loc;
-                    const int d = rem ? owner_of(R, u[k]) : 0;
-                    warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(u[k] - R.part[d]) : 0u,
-                                            (uint64_t)((uint32_t)vv[k] + 1u), wn);
+                    bfs_send_remote<APP>(s, kp, cta, w, imp[k] && !loc, u[k], (uint32_t)vv[k] + 1u, wn);
                 }
             }
 #ifdef ATOS_PROF
@@ -1135,12 +1162,7 @@ __device__ __forceinline__ void pipe_relax(Smem &s, const KParams &kp, int cta, 
         const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
         if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
         warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(st.u[k] - vb), st.nd[k], s.pq_th));
-        if constexpr (MULTI) {
-            const bool rem = imp[k] && !loc;
-            const int d = rem ? owner_of(R, st.u[k]) : 0;
-            warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
-                                    (uint64_t)st.nd[k], wn);
-        }
+        if constexpr (MULTI) bfs_send_remote<APP>(s, kp, cta, w, imp[k] && !loc, st.u[k], st.nd[k], wn);
     }
 }
 
@@ -1220,10 +1242,7 @@ __device__ __forceinline__ void relax_finish(Smem &s, const KParams &kp, int cta
             const bool loc = imp[k] && st.u[k] >= vb && st.u[k] < ve;
             if (wn + 32 > (uint32_t)kWOut) warp_flush_local(s, w, wn, kp.relax_red);
             warp_append_local(s, w, wn, loc, pq_tag((uint32_t)(st.u[k] - vb), st.nd[k], s.pq_th));
-            const bool rem = imp[k] && !loc;
-            const int d = rem ? owner_of(R, st.u[k]) : 0;
-            warp_append_remote<APP>(s, kp, cta, w, rem, d, rem ? (uint32_t)(st.u[k] - R.part[d]) : 0u,
-                                    (uint64_t)st.nd[k], wn);
+            bfs_send_remote<APP>(s, kp, cta, w, imp[k] && !loc, st.u[k], st.nd[k], wn);
         }
     }
 }

@@ -121,9 +121,14 @@ def test_repeated_solves_on_one_handle_and_device_outputs():
         assert st["pops"] >= int((out >= 0).sum())
 
 
+@pytest.mark.parametrize("ratom", [True, False])
 @pytest.mark.parametrize("vr", [2, 3, 4, 8])
 @pytest.mark.parametrize("agg", [0, 1])
-def test_virtual_ranks_identical(vr, agg):
+def test_virtual_ranks_identical(vr, agg, ratom, monkeypatch):
+    # ratom: the sender lowers the owner's depth word and sends activations (the virtual-rank
+    # default); else depth messages the owner applies (the multi-process protocol)
+    if not ratom:
+        monkeypatch.setenv("ATOS_BFS_NORATOM", "1")
     g = inputs.rmat(15, 16, 1, symmetric=True)
     rp, col = g.numpy()
     src = inputs.bfs_sources(g, 1)[0]
