@@ -1,6 +1,6 @@
 # final round-2 evidence pass: GPU tests, smoke, bench (N=1), reference arm, launch list, ncu of the
 # BFS + PR workers (summaries made on the box; only the RMAT-24 BFS report is brought back: <= 64 MiB)
-T=${1:-r2z}
+T=${1:-r2z2}
 mkdir -p gpurun_out/$T
 nproc > gpurun_out/$T/host.txt; lscpu | grep -E "Model name|^CPU\(s\)|Thread|Socket" >> gpurun_out/$T/host.txt
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv >> gpurun_out/$T/host.txt
