@@ -87,6 +87,9 @@ struct alignas(16) BRec {
     uint32_t len;    // long row: edges in the row (piece); short row: unused
 };
 constexpr int kLong = 64;            // rows of >= kLong edges are expanded as aligned chunks of kLongG x kCh1 edges
+// (a batch's short rows -- up to kThreads rows of < kLong edges -- must fit the per-batch edge map
+// of kBitW x 32 edges; kLong = 128 measured RMAT-24 2.425 -> 2.395 ms but overflows it)
+static_assert((int64_t)(kLong - 1) * kThreads <= kBitE, "short rows of a batch must fit the edge map");
 constexpr int kCh1 = 128;            // edges per warp chunk in atos_bfs1.cuh (32 lanes x 4)
 #ifndef ATOS_LONGG
 #define ATOS_LONGG 1
